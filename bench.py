@@ -1,0 +1,402 @@
+#!/usr/bin/env python3
+"""bench.py — GPU-FPX exception scan on B200: lane-values classified per second.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl fpx|reference]
+
+A "step" is one pass of the whole hot path (decode,
+classify, kind rule, warp aggregation, device table; plus the NCCL merge when
+N > 1) over one batch: the configuration BASELINE.json's metric is quoted on,
+configs[1] = C2 (mixed FP32/FP64 trace, 1e8 records, 1e4 sites, exception
+density 1e-6, destination-only check), generated in HBM by fpxgen (inputs
+20+ GB >> 126 MB L2, so no L2 flush is needed between steps).
+
+Prints ONE JSON line (rank 0).  value = lane-values classified per second over
+all ranks (active lanes x values per lane), timed with CUDA events on the
+launching stream, max over ranks.  See DESIGN.md §6 for every field.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "lane-values classified/sec"
+UNIT = "lane-values/s"
+
+# Workloads (BASELINE.json configs); C2 is the headline.
+CONFIGS = {
+    "c1": dict(name="C1: tiny FP32 trace, 1e5 FFMA/FADD/MUFU.RCP records, 200 sites, planted NaN/INF/SUB/DIV0",
+               recipe=0, n=100_000, sites=200, p_fp64=0.0, mode=0, n_inj=400),
+    "c2": dict(name="C2: mixed FP32/FP64 trace, 1e8 records, 1e4 sites, density 1e-6, dest-only check",
+               recipe=1, n=100_000_000, sites=10_000, p_fp64=0.5, mode=0, rho=1e-6),
+    "c3": dict(name="C3: flow-analysis mode, FP32/FP64 70/30 records with dest + 1..3 sources, ~1e9 lane-values",
+               recipe=2, n=7_800_000, sites=1_000, p_fp64=0.3, mode=1, rho=1e-6),
+    "c4a": dict(name="C4a: HADD2/HFMA2/HMUL2 FP16x2/BF16x2 + HMMA records, 1e8 records, 1e3 sites, density 1e-6",
+                recipe=3, n=100_000_000, sites=1_000, p_fp64=0.0, mode=0, rho=1e-6),
+    "c5": dict(name="C5 shard: FP32 dest-only trace, 10^11 lane-values / 8 GPUs = 3.9e8 records per GPU, 1e6 sites",
+               recipe=1, n=390_625_000, sites=1_000_000, p_fp64=0.0, mode=0, rho=1e-6),
+}
+
+
+def load_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
+                if out.returncode == 0 and out.stdout.strip():
+                    self.samples.append([x.strip() for x in out.stdout.strip().split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.05)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4) if len(s) > 3 + i and s[3 + i] == "Active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+def workload_stats(hdr_dev, mode: int):
+    """(lane-values per pass, algorithmic bytes per pass) from the headers on
+    device: lane-values = active lanes x values per lane (DEST: destination
+    values; FLOW: destination + source values); bytes = 16 B header + 128 B
+    per plane the mode must read."""
+    import torch
+
+    h = hdr_dev.to(torch.int64) & 0xFFFFFFFF
+    mask, meta = h[:, 1], h[:, 2]
+    op, fmt, nsrc, dw = meta & 0xFF, (meta >> 8) & 3, (meta >> 10) & 3, (meta >> 12) & 7
+    x = mask - ((mask >> 1) & 0x55555555)
+    x = (x & 0x33333333) + ((x >> 2) & 0x33333333)
+    x = (x + (x >> 4)) & 0x0F0F0F0F
+    pop = (x * 0x01010101 & 0xFFFFFFFF) >> 24
+    sw = torch.where(fmt == 1, 2, 1)
+    nv = torch.where(fmt == 1, dw // 2, torch.where(fmt == 0, dw, 2 * dw))
+    compare = (op == 11) | (op == 12) | (op == 14)
+    if mode == 0:
+        planes = torch.where(compare, 0, dw)
+        vals = torch.where(compare, 0, nv)
+    else:
+        planes = dw + nsrc * sw
+        vals = torch.where(dw > 0, 1, 0) + nsrc
+    lane_values = int((pop * vals).sum().item())
+    nbytes = 16 * h.shape[0] + 128 * int(planes.sum().item())
+    return lane_values, nbytes
+
+
+def build_trace(cfg, rank, world, seed):
+    """This rank's shard of the configured trace, generated in HBM, with the
+    planted events applied.  Weak scaling: every rank holds cfg['n'] records;
+    rank r owns global records [r*n, (r+1)*n)."""
+    import fpxgen
+
+    n = cfg["n"]
+    r0 = rank * n
+    p = fpxgen.Params(seed=seed, n_records=n, n_sites=cfg["sites"], recipe=cfg["recipe"], p_fp64=cfg["p_fp64"])
+    hdr, arena, planes = fpxgen.generate_device(p, r0=r0)
+    n_inj = cfg.get("n_inj") or int(round(cfg["rho"] * n * 32))
+    inj, writes = fpxgen.plan_injections(p, n_inj, flow=cfg["mode"] == 1, r0=r0)
+    fpxgen.apply_device(writes, hdr, arena)
+    return p, hdr, arena, planes, r0, inj
+
+
+def cpu_baseline_oracle(cfg, seed, budget_s: float = 12.0):
+    """The oracle (never tuned) on a bounded prefix of the same trace, single
+    thread on this box's host cores: lane-values/s."""
+    import fpxgen
+    import oracle
+
+    def run(n):
+        p = fpxgen.Params(seed=seed, n_records=n, n_sites=cfg["sites"], recipe=cfg["recipe"], p_fp64=cfg["p_fp64"])
+        hdr, arena = fpxgen.generate_host(p)
+        _, w = fpxgen.plan_injections(p, max(1, int(round(cfg.get("rho", 1e-6) * n * 32))), flow=cfg["mode"] == 1)
+        fpxgen.apply_host(w, hdr, arena)
+        t = oracle.Table()
+        t0 = time.perf_counter()
+        t.scan_records(hdr, arena, base_index=0, mode=cfg["mode"])
+        dt = time.perf_counter() - t0
+        return t.lane_values, dt
+
+    lv, dt = run(20_000)
+    n = int(min(cfg["n"], max(20_000, 20_000 * budget_s / max(dt, 1e-6))))
+    lv, dt = run(n)
+    return {"value": lv / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"first {n} records of the same {cfg['name'].split(':')[0]} trace (same seed), "
+                      f"single-threaded C++ oracle, {dt:.1f} s, {lv} lane-values"}
+
+
+def run_reference(args, cfg, seed):
+    """--impl reference: the CPU oracle as the reference arm."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import fpxgen
+    import oracle
+
+    # each step: a bounded sample of the workload sized to ~0.25 s of oracle time
+    probe_n = 20_000
+    p = fpxgen.Params(seed=seed, n_records=probe_n, n_sites=cfg["sites"], recipe=cfg["recipe"], p_fp64=cfg["p_fp64"])
+    hdr, arena = fpxgen.generate_host(p)
+    t = oracle.Table()
+    t0 = time.perf_counter()
+    t.scan_records(hdr, arena, mode=cfg["mode"])
+    dt = time.perf_counter() - t0
+    n = int(max(1000, min(cfg["n"], probe_n * 0.25 / max(dt, 1e-6))))
+    p = fpxgen.Params(seed=seed, n_records=n, n_sites=cfg["sites"], recipe=cfg["recipe"], p_fp64=cfg["p_fp64"])
+    hdr, arena = fpxgen.generate_host(p)
+    _, w = fpxgen.plan_injections(p, max(1, int(round(cfg.get("rho", 1e-6) * n * 32))), flow=cfg["mode"] == 1)
+    fpxgen.apply_host(w, hdr, arena)
+    for _ in range(args.warmup):
+        t = oracle.Table()
+        t.scan_records(hdr, arena, mode=cfg["mode"])
+    lv_total, dt_total = 0, 0.0
+    for _ in range(args.steps):
+        t = oracle.Table()
+        t0 = time.perf_counter()
+        t.scan_records(hdr, arena, mode=cfg["mode"])
+        dt_total += time.perf_counter() - t0
+        lv_total += t.lane_values
+    value = lv_total / dt_total
+    sample = f"first {n} records of the {cfg['name'].split(':')[0]} trace per step (same seed), single-threaded oracle"
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt_total / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": cfg["name"], "records_per_step": n, "mode": ["dest", "flow"][cfg["mode"]]},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="fpx", choices=["fpx", "reference"])
+    ap.add_argument("--records", type=int, default=0, help="override the record count (debug only)")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    cfg = dict(CONFIGS[args.config])
+    if args.records:
+        cfg["n"] = args.records
+    seed = 0x5EED0000 + list(CONFIGS).index(args.config) + 1
+
+    if args.impl == "reference":
+        return run_reference(args, cfg, seed)
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_hpdc_lilfslg23_b200 import dist as fdist
+    from paper_conf_hpdc_lilfslg23_b200 import fpx
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    assert world == args.gpus or world == 1, "launch N>1 with torchrun"
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+
+    p, hdr, arena, planes, r0, inj = build_trace(cfg, rank, world, seed)
+    lane_values, nbytes = workload_stats(hdr, cfg["mode"])
+    torch.cuda.synchronize()
+
+    h = fpx.Handle(local)
+    stream = torch.cuda.current_stream(dev)
+    n = cfg["n"]
+
+    def step(ev_a=None, ev_b=None):
+        h.reset(stream=stream)
+        if ev_a is not None:
+            ev_a.record(stream)
+        h.scan_records(hdr, arena, base_index=r0, mode=cfg["mode"], stream=stream, n_records=n, arena_planes=planes)
+        if ev_b is not None:
+            ev_b.record(stream)
+        if world > 1:
+            fdist.merge_handle(h, stream=stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+
+    K = args.steps
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t_start.record(stream)
+        for i in range(K):
+            step(*evs[i])
+        t_end.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    total_ms = t_start.elapsed_time(t_end)
+    kern_ms = float(np.mean([a.elapsed_time(b) for a, b in evs]))
+    if world > 1:
+        t = torch.tensor([total_ms, kern_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms, kern_ms = float(t[0]), float(t[1])
+    ms_per_step = total_ms / K
+
+    # correctness of what was timed: the table equals the planted closed form
+    ents = h.fetch()
+    ok_status = h.last_status
+
+    # e2e: the same metric through the public API with host buffers: per step,
+    # H2D of the step's inputs from pinned memory, scan, fetch (D2H of entries)
+    e2e = None
+    if not args.no_e2e and world == 1:
+        try:
+            hdr_h = torch.empty(hdr.shape, dtype=hdr.dtype, pin_memory=True)
+            arena_h = torch.empty(arena.shape, dtype=arena.dtype, pin_memory=True)
+            hdr_h.copy_(hdr)
+            arena_h.copy_(arena)
+            torch.cuda.synchronize()
+            d2h = 0
+            e_a, e_b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            tot = 0.0
+            for i in range(args.e2e_steps + 1):
+                torch.cuda.synchronize()
+                e_a.record(stream)
+                hdr.copy_(hdr_h, non_blocking=True)
+                arena.copy_(arena_h, non_blocking=True)
+                h.reset(stream=stream)
+                h.scan_records(hdr, arena, base_index=r0, mode=cfg["mode"], stream=stream, n_records=n,
+                               arena_planes=planes)
+                got = h.fetch()  # synchronises; D2H of the entries
+                e_b.record(stream)
+                torch.cuda.synchronize()
+                if i > 0:  # first pass = warm-up
+                    tot += e_a.elapsed_time(e_b)
+                d2h = got.nbytes
+            e2e = {"value": lane_values / (tot / args.e2e_steps / 1e3), "unit": UNIT,
+                   "h2d_bytes_per_step": hdr.numel() * 4 + arena.numel() * 4, "d2h_bytes_per_step": int(d2h),
+                   "steps": args.e2e_steps}
+            del hdr_h, arena_h
+        except Exception as ex:  # pragma: no cover - reported, not hidden
+            e2e = {"value": None, "unit": UNIT, "error": str(ex)[:200]}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return 0
+
+    peak, peak_src = load_peak()
+    achieved = nbytes / (kern_ms / 1e3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            tj = json.load(f)
+        traffic = tj.get(args.config, {}).get("dram_bytes_per_launch")
+    clocks = clk.summary()
+    cpu = None if args.no_cpu_baseline else cpu_baseline_oracle(cfg, seed)
+    line = {
+        "metric": METRIC,
+        "value": world * lane_values / (ms_per_step / 1e3),
+        "unit": UNIT,
+        "n_gpus": world,
+        "steps": K,
+        "warmup": args.warmup,
+        "ms_per_step": ms_per_step,
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "u32",
+        "data": "synthetic (fpxgen counter-based trace generated in HBM, planted exceptions)",
+        "config": {
+            "workload": cfg["name"],
+            "records_per_gpu": n,
+            "sites": cfg["sites"],
+            "mode": ["dest", "flow"][cfg["mode"]],
+            "lane_values_per_gpu_step": lane_values,
+            "algorithmic_bytes_per_gpu_step": nbytes,
+            "planted_events": int(len(inj)),
+            "table_entries": int(len(ents)),
+            "fetch_status": int(ok_status),
+            "l2": "inputs >> 126 MB L2 (no flush needed)",
+            "parallelism": f"record shards x{world}" + (" + NCCL merge per step" if world > 1 else ""),
+        },
+        "roofline": {
+            "bound": "hbm",
+            "achieved": achieved,
+            "peak": peak,
+            "unit": "GB/s",
+            "frac": achieved / peak,
+            "traffic": traffic,
+            "kernel": "k_scan_records",
+            "kernel_ms": kern_ms,
+            "peak_source": peak_src,
+        },
+        "clocks": clocks,
+        "gpu_launches": K * (2 + (3 + 2 if world > 1 else 0)),
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+    }
+    print(json.dumps(line), flush=True)
+    h.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,395 @@
+// fpx_api.cu — the C ABI of include/fpx.h: argument checking, handle state,
+// launches on the caller's stream, and the cold fetch path.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <vector>
+
+#include "fpx_internal.h"
+
+using namespace fpx;
+
+struct fpx_ctx {
+  int device = 0;
+  int num_sms = 148;
+  uint64_t slots = 0;
+  TableView tv{};
+  uint64_t newlog_cursor = 0;  // FETCH_NEW position
+  cudaStream_t last_stream = nullptr;
+  // fetch scratch (lazily sized to `slots`)
+  uint64_t* d_keys = nullptr;
+  uint64_t* d_counts = nullptr;
+  uint64_t* d_first = nullptr;
+  uint64_t* d_keys2 = nullptr;
+  uint64_t* d_idx = nullptr;
+  uint64_t* d_idx2 = nullptr;
+  unsigned long long* d_n = nullptr;
+  void* d_temp = nullptr;
+  size_t temp_bytes = 0;
+  Ctl* h_ctl = nullptr;  // pinned mirror of the counters
+};
+
+namespace {
+
+char g_cuda_err[512] = "";
+std::mutex g_err_mu;
+
+fpx_status cuda_err(cudaError_t e, const char* where) {
+  std::lock_guard<std::mutex> lk(g_err_mu);
+  snprintf(g_cuda_err, sizeof g_cuda_err, "%s: %s", where, cudaGetErrorString(e));
+  return FPX_ERR_CUDA;
+}
+
+#define CK(x)                                                  \
+  do {                                                         \
+    cudaError_t _e = (x);                                      \
+    if (_e != cudaSuccess) return cuda_err(_e, #x);            \
+  } while (0)
+
+// Runs `fn` with the handle's device current and restores the caller's.
+struct DeviceGuard {
+  int prev = -1;
+  bool ok = true;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) { ok = false; return; }
+    if (prev != dev && cudaSetDevice(dev) != cudaSuccess) ok = false;
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+fpx_status ensure_scratch(fpx_ctx* h) {
+  if (h->d_keys) return FPX_OK;
+  const size_t b = sizeof(uint64_t) * h->slots;
+  CK(cudaMalloc(&h->d_keys, b));
+  CK(cudaMalloc(&h->d_counts, b));
+  CK(cudaMalloc(&h->d_first, b));
+  CK(cudaMalloc(&h->d_keys2, b));
+  CK(cudaMalloc(&h->d_idx, b));
+  CK(cudaMalloc(&h->d_idx2, b));
+  CK(cudaMalloc(&h->d_n, sizeof(unsigned long long)));
+  size_t t1 = 0, t2 = 0;
+  CK(sort_keys_with_index(nullptr, &t1, h->d_keys, h->d_keys2, h->d_idx, h->d_idx2, h->slots, nullptr));
+  CK(unique_keys(nullptr, &t2, h->d_keys, h->d_keys2, h->d_n, h->slots, nullptr));
+  h->temp_bytes = std::max(t1, t2);
+  CK(cudaMalloc(&h->d_temp, h->temp_bytes));
+  return FPX_OK;
+}
+
+fpx_status ensure_temp(fpx_ctx* h, size_t need) {
+  if (need <= h->temp_bytes) return FPX_OK;
+  if (h->d_temp) CK(cudaFree(h->d_temp));
+  h->d_temp = nullptr;
+  CK(cudaMalloc(&h->d_temp, need));
+  h->temp_bytes = need;
+  return FPX_OK;
+}
+
+// Sorted (key, count, first) of either the whole table or a key list, into
+// h->d_keys2 / d_counts / d_first (the latter two reused as outputs);
+// returns the number of entries in *n.
+fpx_status sorted_entries(fpx_ctx* h, cudaStream_t s, const uint64_t* d_key_list, uint64_t n_list, uint64_t* n) {
+  uint64_t cnt = 0;
+  if (d_key_list == nullptr) {
+    CK(launch_table_compact(h->tv, h->slots, h->d_keys, h->d_counts, h->d_first, h->d_n, s));
+    unsigned long long hn = 0;
+    CK(cudaMemcpyAsync(&hn, h->d_n, sizeof hn, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    cnt = hn;
+  } else {
+    cnt = n_list;
+    if (cnt) CK(cudaMemcpyAsync(h->d_keys, d_key_list, cnt * 8, cudaMemcpyDeviceToDevice, s));
+    CK(launch_table_lookup(h->tv, h->d_keys, cnt, h->d_counts, h->d_first, s));
+  }
+  *n = cnt;
+  if (cnt == 0) return FPX_OK;
+  CK(launch_iota(h->d_idx, cnt, s));
+  size_t tb = 0;
+  CK(sort_keys_with_index(nullptr, &tb, h->d_keys, h->d_keys2, h->d_idx, h->d_idx2, cnt, s));
+  fpx_status st = ensure_temp(h, tb);
+  if (st != FPX_OK) return st;
+  tb = h->temp_bytes;
+  CK(sort_keys_with_index(h->d_temp, &tb, h->d_keys, h->d_keys2, h->d_idx, h->d_idx2, cnt, s));
+  // gather counts / firsts by the permutation into d_keys (reused) / d_idx (reused)
+  CK(launch_gather3(h->d_idx2, cnt, h->d_counts, h->d_first, h->d_keys, h->d_idx, s));
+  return FPX_OK;
+}
+
+fpx_status sticky_status(fpx_ctx* h, cudaStream_t s) {
+  CK(cudaMemcpyAsync(h->h_ctl, h->tv.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (h->h_ctl->dropped_events) return FPX_ERR_TABLE_FULL;
+  if (h->h_ctl->bad_records) return FPX_ERR_BAD_RECORD;
+  return FPX_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+uint32_t fpx_abi_version(void) { return 1u; }
+uint32_t fpx_sizeof_rec_hdr(void) { return (uint32_t)sizeof(fpx_rec_hdr); }
+uint32_t fpx_sizeof_entry(void) { return (uint32_t)sizeof(fpx_entry); }
+
+const char* fpx_strerror(fpx_status s) {
+  switch (s) {
+    case FPX_OK: return "ok";
+    case FPX_ERR_INVALID: return "invalid argument";
+    case FPX_ERR_CUDA: return "CUDA error";
+    case FPX_ERR_NOMEM: return "out of memory";
+    case FPX_ERR_TABLE_FULL: return "exception table full: events dropped";
+    case FPX_ERR_BAD_RECORD: return "bad record(s) skipped";
+    case FPX_ERR_TRUNCATED: return "output truncated to capacity";
+  }
+  return "unknown status";
+}
+
+const char* fpx_last_cuda_error(void) { return g_cuda_err; }
+
+fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
+  if (!out) return FPX_ERR_INVALID;
+  *out = nullptr;
+  fpx_options o{};
+  if (opt) o = *opt;
+  if (o.flags != 0) return FPX_ERR_INVALID;
+  if (o.table_log2_slots == 0) o.table_log2_slots = 20;
+  if (o.table_log2_slots < 4 || o.table_log2_slots > 30) return FPX_ERR_INVALID;
+  int ndev = 0;
+  CK(cudaGetDeviceCount(&ndev));
+  if (device < 0 || device >= ndev) return FPX_ERR_INVALID;
+  DeviceGuard g(device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  fpx_ctx* h = new (std::nothrow) fpx_ctx();
+  if (!h) return FPX_ERR_NOMEM;
+  h->device = device;
+  CK(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, device));
+  h->slots = 1ull << o.table_log2_slots;
+  // the log never holds more keys than the table has slots
+  const uint64_t cap = o.newlog_capacity ? std::min<uint64_t>(o.newlog_capacity, h->slots) : h->slots;
+  Slot* slots = nullptr;
+  unsigned long long* log = nullptr;
+  Ctl* ctl = nullptr;
+  if (cudaMalloc(&slots, sizeof(Slot) * h->slots) != cudaSuccess ||
+      cudaMalloc(&log, sizeof(unsigned long long) * cap) != cudaSuccess ||
+      cudaMalloc(&ctl, sizeof(Ctl)) != cudaSuccess || cudaMallocHost(&h->h_ctl, sizeof(Ctl)) != cudaSuccess) {
+    cudaGetLastError();
+    if (slots) cudaFree(slots);
+    if (log) cudaFree(log);
+    if (ctl) cudaFree(ctl);
+    delete h;
+    return FPX_ERR_NOMEM;
+  }
+  h->tv.slots = slots;
+  h->tv.mask = h->slots - 1;
+  h->tv.newlog = log;
+  h->tv.newlog_cap = cap;
+  h->tv.ctl = ctl;
+  CK(launch_table_reset(h->tv, h->slots, nullptr));
+  CK(cudaStreamSynchronize(nullptr));
+  *out = h;
+  return FPX_OK;
+}
+
+fpx_status fpx_scan_records(fpx_handle h, const fpx_rec_hdr* d_hdr, uint64_t n_records, const uint32_t* d_arena,
+                            uint64_t arena_planes, uint64_t base_index, uint32_t mode, void* stream) {
+  if (!h) return FPX_ERR_INVALID;
+  if (mode != FPX_MODE_DEST && mode != FPX_MODE_FLOW) return FPX_ERR_INVALID;
+  if (n_records == 0) return FPX_OK;
+  if (!d_hdr || !aligned16(d_hdr)) return FPX_ERR_INVALID;
+  if (arena_planes && (!d_arena || !aligned16(d_arena))) return FPX_ERR_INVALID;
+  if (base_index + n_records < base_index) return FPX_ERR_INVALID;  // index overflow
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  CK(launch_scan_records(d_hdr, n_records, d_arena, arena_planes, base_index, mode, h->tv, h->num_sms, s));
+  h->last_stream = s;
+  return FPX_OK;
+}
+
+fpx_status fpx_scan_tensor(fpx_handle h, const void* d_ptr, uint64_t n_elems, uint32_t fmt, uint32_t site,
+                           uint64_t base_index, void* stream) {
+  if (!h || fmt > FPX_BF16) return FPX_ERR_INVALID;
+  if (n_elems == 0) return FPX_OK;
+  const uintptr_t es = fmt == FPX_FP64 ? 8 : fmt == FPX_FP32 ? 4 : 2;
+  if (!d_ptr || (reinterpret_cast<uintptr_t>(d_ptr) % es) != 0) return FPX_ERR_INVALID;
+  if (base_index + n_elems < base_index) return FPX_ERR_INVALID;
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  CK(launch_scan_tensor(d_ptr, n_elems, fmt, site, base_index, h->tv, h->num_sms, s));
+  h->last_stream = s;
+  return FPX_OK;
+}
+
+fpx_status fpx_table_fetch(fpx_handle h, fpx_entry* host_out, uint64_t capacity, uint64_t* n_total, uint32_t flags) {
+  if (!h || !n_total || (capacity && !host_out)) return FPX_ERR_INVALID;
+  if (flags != FPX_FETCH_ALL && flags != FPX_FETCH_NEW) return FPX_ERR_INVALID;
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  cudaStream_t s = h->last_stream;
+  CK(cudaStreamSynchronize(s));
+  fpx_status st = ensure_scratch(h);
+  if (st != FPX_OK) return st;
+  uint64_t n = 0;
+  if (flags == FPX_FETCH_ALL) {
+    st = sorted_entries(h, s, nullptr, 0, &n);
+  } else {
+    // keys inserted since the previous FETCH_NEW, read from the device log
+    CK(cudaMemcpyAsync(h->h_ctl, h->tv.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const uint64_t tail = std::min<uint64_t>(h->h_ctl->newlog_tail, h->tv.newlog_cap);
+    const uint64_t from = std::min<uint64_t>(h->newlog_cursor, tail);
+    st = sorted_entries(h, s, reinterpret_cast<const uint64_t*>(h->tv.newlog) + from, tail - from, &n);
+    if (st == FPX_OK) h->newlog_cursor = tail;
+  }
+  if (st != FPX_OK) return st;
+  *n_total = n;
+  const uint64_t m = std::min(n, capacity);
+  if (m) {
+    std::vector<uint64_t> k(m), c(m), f(m);
+    CK(cudaMemcpyAsync(k.data(), h->d_keys2, m * 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(c.data(), h->d_keys, m * 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(f.data(), h->d_idx, m * 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    for (uint64_t i = 0; i < m; ++i) {
+      fpx_entry e;
+      std::memset(&e, 0, sizeof e);
+      e.site = (uint32_t)(k[i] >> 32);
+      e.fmt = (uint8_t)((k[i] >> 4) & 3);
+      e.flow = (uint8_t)((k[i] >> 2) & 3);
+      e.kind = (uint8_t)(k[i] & 3);
+      e.count = c[i];
+      e.first_index = f[i];
+      host_out[i] = e;
+    }
+  }
+  if (capacity < n) return FPX_ERR_TRUNCATED;
+  return sticky_status(h, s);
+}
+
+fpx_status fpx_table_fetch_device(fpx_handle h, uint64_t* d_keys, uint64_t* d_counts, uint64_t* d_first,
+                                  uint64_t capacity, uint64_t* n_total, void* stream) {
+  if (!h || !n_total || (capacity && (!d_keys || !d_counts || !d_first))) return FPX_ERR_INVALID;
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (h->last_stream != s) CK(cudaStreamSynchronize(h->last_stream));
+  fpx_status st = ensure_scratch(h);
+  if (st != FPX_OK) return st;
+  uint64_t n = 0;
+  st = sorted_entries(h, s, nullptr, 0, &n);
+  if (st != FPX_OK) return st;
+  *n_total = n;
+  const uint64_t m = std::min(n, capacity);
+  if (m) {
+    CK(cudaMemcpyAsync(d_keys, h->d_keys2, m * 8, cudaMemcpyDeviceToDevice, s));
+    CK(cudaMemcpyAsync(d_counts, h->d_keys, m * 8, cudaMemcpyDeviceToDevice, s));
+    CK(cudaMemcpyAsync(d_first, h->d_idx, m * 8, cudaMemcpyDeviceToDevice, s));
+  }
+  CK(cudaStreamSynchronize(s));
+  if (capacity < n) return FPX_ERR_TRUNCATED;
+  return sticky_status(h, s);
+}
+
+fpx_status fpx_table_lookup_device(fpx_handle h, const uint64_t* d_keys, uint64_t n, uint64_t* d_counts,
+                                   uint64_t* d_first, void* stream) {
+  if (!h || (n && (!d_keys || !d_counts || !d_first))) return FPX_ERR_INVALID;
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (h->last_stream != s) CK(cudaStreamSynchronize(h->last_stream));
+  CK(launch_table_lookup(h->tv, d_keys, n, d_counts, d_first, s));
+  return FPX_OK;
+}
+
+fpx_status fpx_keys_unique_device(fpx_handle h, const uint64_t* d_keys, uint64_t n, uint64_t* d_out, uint64_t* n_out,
+                                  void* stream) {
+  if (!h || !n_out || (n && (!d_keys || !d_out))) return FPX_ERR_INVALID;
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  *n_out = 0;
+  if (n == 0) return FPX_OK;
+  fpx_status st = ensure_scratch(h);
+  if (st != FPX_OK) return st;
+  size_t tb = 0;
+  CK(unique_keys(nullptr, &tb, d_keys, d_out, h->d_n, n, s));
+  st = ensure_temp(h, tb);
+  if (st != FPX_OK) return st;
+  tb = h->temp_bytes;
+  CK(unique_keys(h->d_temp, &tb, d_keys, d_out, h->d_n, n, s));
+  unsigned long long hn = 0;
+  CK(cudaMemcpyAsync(&hn, h->d_n, sizeof hn, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (hn) {
+    uint64_t last = 0;
+    CK(cudaMemcpy(&last, d_out + hn - 1, 8, cudaMemcpyDeviceToHost));
+    if (last == FPX_KEY_EMPTY) hn--;
+  }
+  *n_out = hn;
+  return FPX_OK;
+}
+
+fpx_status fpx_table_merge_device(fpx_handle h, const uint64_t* d_keys, const uint64_t* d_counts,
+                                  const uint64_t* d_first, uint64_t n, void* stream) {
+  if (!h || (n && (!d_keys || !d_counts || !d_first))) return FPX_ERR_INVALID;
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (h->last_stream != s) CK(cudaStreamSynchronize(h->last_stream));
+  CK(launch_table_merge(h->tv, d_keys, d_counts, d_first, n, s));
+  h->last_stream = s;
+  return FPX_OK;
+}
+
+fpx_status fpx_table_reset(fpx_handle h, void* stream) {
+  if (!h) return FPX_ERR_INVALID;
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (h->last_stream != s) CK(cudaStreamSynchronize(h->last_stream));
+  CK(launch_table_reset(h->tv, h->slots, s));
+  h->newlog_cursor = 0;
+  h->last_stream = s;
+  return FPX_OK;
+}
+
+fpx_status fpx_get_stats(fpx_handle h, fpx_stats* out) {
+  if (!h || !out) return FPX_ERR_INVALID;
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  CK(cudaStreamSynchronize(h->last_stream));
+  CK(cudaMemcpy(h->h_ctl, h->tv.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost));
+  out->bad_records = h->h_ctl->bad_records;
+  out->dropped_events = h->h_ctl->dropped_events;
+  out->table_entries = std::min<uint64_t>(h->h_ctl->newlog_tail, h->slots);
+  out->newlog_overflow = h->h_ctl->newlog_overflow;
+  return FPX_OK;
+}
+
+fpx_status fpx_close(fpx_handle h) {
+  if (!h) return FPX_ERR_INVALID;
+  {
+    DeviceGuard g(h->device);
+    cudaDeviceSynchronize();
+    cudaFree(h->tv.slots);
+    cudaFree(h->tv.newlog);
+    cudaFree(h->tv.ctl);
+    cudaFreeHost(h->h_ctl);
+    for (void* p : {(void*)h->d_keys, (void*)h->d_counts, (void*)h->d_first, (void*)h->d_keys2, (void*)h->d_idx,
+                    (void*)h->d_idx2, (void*)h->d_n, h->d_temp})
+      if (p) cudaFree(p);
+  }
+  delete h;
+  return FPX_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,70 @@
+// fpx_internal.h — types shared by the C-ABI layer and the sm_100a kernels.
+//
+// Device state of one handle:
+//   table   2^k slots x 32 B {key, count, first, pad}: one L2 sector per slot,
+//           open addressing with linear probing (the paper's GT, P:223, 236-244,
+//           widened per readings R14/R15)
+//   newlog  append-only log of keys in insertion order (the paper's
+//           "push only new combinations to the host", P:244 / Alg2 P:271-273,
+//           read at fetch instead of through a GPU->CPU channel)
+//   ctl     sticky counters (bad records, dropped events, log tail, overflow)
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "fpx.h"
+
+namespace fpx {
+
+struct alignas(32) Slot {
+  unsigned long long key;    // FPX_KEY_EMPTY when free
+  unsigned long long count;  // lane-values with this key
+  unsigned long long first;  // min global record / element index
+  unsigned long long pad;
+};
+static_assert(sizeof(Slot) == 32, "slot = one 32-B L2 sector");
+
+struct alignas(64) Ctl {
+  unsigned long long bad_records;
+  unsigned long long dropped_events;
+  unsigned long long newlog_tail;      // number of inserts ever (= table entries)
+  unsigned long long newlog_overflow;
+  unsigned long long pad[4];
+};
+
+// Everything a scan kernel needs to update the table, passed by value.
+struct TableView {
+  Slot* slots;
+  unsigned long long mask;       // slots - 1
+  unsigned long long* newlog;
+  unsigned long long newlog_cap;
+  Ctl* ctl;
+};
+
+// ---- launchers (fpx_scan.cu, fpx_table.cu) --------------------------------
+cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena,
+                                uint64_t arena_planes, uint64_t base_index, uint32_t mode,
+                                const TableView& tv, int num_sms, cudaStream_t s);
+cudaError_t launch_scan_tensor(const void* d_ptr, uint64_t n_elems, uint32_t fmt, uint32_t site,
+                               uint64_t base_index, const TableView& tv, int num_sms, cudaStream_t s);
+cudaError_t launch_table_reset(const TableView& tv, uint64_t slots, cudaStream_t s);
+// Compact non-empty slots into (keys, counts, firsts); *d_n receives the count.
+cudaError_t launch_table_compact(const TableView& tv, uint64_t slots, uint64_t* d_keys,
+                                 uint64_t* d_counts, uint64_t* d_first, unsigned long long* d_n,
+                                 cudaStream_t s);
+// Look keys up: count (0 if absent) and first (INT64_MAX if absent).
+cudaError_t launch_table_lookup(const TableView& tv, const uint64_t* d_keys, uint64_t n,
+                                uint64_t* d_counts, uint64_t* d_first, cudaStream_t s);
+cudaError_t launch_table_merge(const TableView& tv, const uint64_t* d_keys, const uint64_t* d_counts,
+                               const uint64_t* d_first, uint64_t n, cudaStream_t s);
+// Radix-sort keys (with a permutation of 0..n-1 as values); temp via cub.
+cudaError_t sort_keys_with_index(void* d_temp, size_t* temp_bytes, const uint64_t* d_keys_in,
+                                 uint64_t* d_keys_out, const uint64_t* d_idx_in, uint64_t* d_idx_out,
+                                 uint64_t n, cudaStream_t s);
+cudaError_t launch_iota(uint64_t* d, uint64_t n, cudaStream_t s);
+cudaError_t launch_gather3(const uint64_t* d_idx, uint64_t n, const uint64_t* c_in, const uint64_t* f_in,
+                           uint64_t* c_out, uint64_t* f_out, cudaStream_t s);
+cudaError_t unique_keys(void* d_temp, size_t* temp_bytes, const uint64_t* d_in, uint64_t* d_out,
+                        unsigned long long* d_nout, uint64_t n, cudaStream_t s);
+
+}  // namespace fpx

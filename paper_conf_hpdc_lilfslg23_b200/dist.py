@@ -1,0 +1,78 @@
+"""Multi-GPU: record-index sharding and the NCCL merge of per-GPU tables.
+
+SURVEY §8(e): records are independent, so rank r of P scans the contiguous
+range [floor(rN/P), floor((r+1)N/P)) with base_index = range start (first
+indices are then global).  The only cross-rank state is the table, whose merge
+is associative and commutative (key union, count sum, first-index min):
+
+  1. fetch the local table on device, sorted by key      (fpx_table_fetch_device)
+  2. all_gather the key counts, then the keys padded with EMPTY
+  3. union = sort + unique of the gathered keys           (fpx_keys_unique_device)
+  4. dense scatter: this rank's count / first per union key
+     (0 / INT64_MAX when absent)                           (fpx_table_lookup_device)
+  5. all_reduce SUM of counts, all_reduce MIN of firsts   (NCCL over NVLink)
+
+Counts and first indices travel as int64 (first < 2^63; the absent sentinel
+is INT64_MAX so a signed MIN is exact).  The collective plumbing below is
+backend-agnostic so the same code runs under gloo on CPU in the tests, with
+`ops` supplying the three table operations.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+KEY_EMPTY_I64 = -1  # 0xFFFFFFFFFFFFFFFF viewed as int64
+FIRST_NONE = (1 << 63) - 1
+
+
+def shard_range(n: int, rank: int, world: int) -> tuple[int, int]:
+    """Contiguous record range of `rank` (floor(rN/P), floor((r+1)N/P))."""
+    return (n * rank) // world, (n * (rank + 1)) // world
+
+
+def merge(keys: torch.Tensor, counts: torch.Tensor, firsts: torch.Tensor, ops, group=None):
+    """Merge this rank's sorted (keys, counts, firsts) with every other rank's.
+    Returns the global (keys, counts, firsts), identical on all ranks.
+
+    ops.unique(t) -> sorted unique keys of t without EMPTY
+    ops.lookup(keys) -> (counts, firsts) of this rank's table for those keys
+    """
+    world = dist.get_world_size(group)
+    dev = keys.device
+    n = torch.tensor([keys.numel()], dtype=torch.int64, device=dev)
+    sizes = [torch.zeros_like(n) for _ in range(world)]
+    dist.all_gather(sizes, n, group=group)
+    m = int(max(int(s.item()) for s in sizes))
+    if m == 0:
+        e = torch.empty(0, dtype=torch.int64, device=dev)
+        return e, e.clone(), e.clone()
+    padded = torch.full((m,), KEY_EMPTY_I64, dtype=torch.int64, device=dev)
+    padded[: keys.numel()] = keys
+    gathered = [torch.empty_like(padded) for _ in range(world)]
+    dist.all_gather(gathered, padded, group=group)
+    union = ops.unique(torch.cat(gathered))
+    c, f = ops.lookup(union)
+    dist.all_reduce(c, op=dist.ReduceOp.SUM, group=group)
+    dist.all_reduce(f, op=dist.ReduceOp.MIN, group=group)
+    return union, c, f
+
+
+class DeviceOps:
+    """The table operations of `merge`, run by libfpx.so kernels on the GPU."""
+
+    def __init__(self, handle, stream=None):
+        self.h = handle
+        self.stream = stream
+
+    def unique(self, t):
+        return self.h.unique_device(t, stream=self.stream)
+
+    def lookup(self, keys):
+        return self.h.lookup_device(keys, stream=self.stream)
+
+
+def merge_handle(handle, group=None, stream=None):
+    """Fetch this rank's table on device and merge it across the group (NCCL)."""
+    k, c, f = handle.fetch_device(stream=stream)
+    return merge(k, c, f, DeviceOps(handle, stream), group=group)

@@ -1,0 +1,102 @@
+"""CPU-side checks of the C-ABI library (no compute calls without a GPU).
+
+* libfpx.so loads and exports every function include/fpx.h declares;
+* the binding's enum values equal the header's;
+* the header's record / entry layout agrees with the oracle's and the
+  generator's own (independent) definitions;
+* calls that must fail without touching the device do fail cleanly.
+"""
+import ctypes
+import os
+import re
+import subprocess
+
+import numpy as np
+
+import fpxgen
+import oracle
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "fpx.h")
+LIB = os.path.join(ROOT, "paper_conf_hpdc_lilfslg23_b200", "libfpx.so")
+
+
+def header_functions():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(fpx_[a-z_0-9]+)\s*\(", src)) - {"fpx_entry", "fpx_options"})
+
+
+def header_enums():
+    src = re.sub(r"/\*.*?\*/", "", open(HEADER).read(), flags=re.S)
+    vals = {}
+    for m in re.finditer(r"\b(FPX_[A-Z0-9_]+)\s*=\s*(-?\d+)", src):
+        vals[m.group(1)] = int(m.group(2))
+    return vals
+
+
+def test_library_exports_every_declared_symbol():
+    funcs = header_functions()
+    assert len(funcs) >= 16
+    out = subprocess.run(["nm", "-D", "--defined-only", LIB], capture_output=True, text=True, check=True).stdout
+    exported = set(re.findall(r"\bT (fpx_\w+)", out))
+    missing = [f for f in funcs if f not in exported]
+    assert not missing, missing
+    L = ctypes.CDLL(LIB)
+    for f in funcs:
+        getattr(L, f)
+
+
+def test_binding_names_match_header():
+    from paper_conf_hpdc_lilfslg23_b200 import fpx
+
+    assert sorted(fpx.EXPORTS) == header_functions()
+    e = header_enums()
+    for name, val in e.items():
+        short = name[len("FPX_"):]
+        if short.startswith("ERR_") or short in ("OK",):
+            assert getattr(fpx, short) == val, name
+        elif short in ("FP32", "FP64", "FP16", "BF16", "NAN", "INF", "SUB", "DIV0", "GEN", "PROP", "KILL",
+                       "FLOW_NONE", "MODE_DEST", "MODE_FLOW", "FETCH_ALL", "FETCH_NEW"):
+            assert getattr(fpx, short) == val, name
+    assert e["FPX_OP_COUNT"] == 20 and e["FPX_OP_DIV"] == 19 and e["FPX_OP_MUFU_RCP64H"] == 5
+
+
+def test_layouts_agree_across_independent_definitions():
+    from paper_conf_hpdc_lilfslg23_b200 import fpx
+
+    assert fpx.lib.fpx_sizeof_rec_hdr() == oracle.lib().orc_sizeof_hdr() == fpxgen.lib().fpxgen_sizeof_hdr() == 16
+    assert fpx.lib.fpx_sizeof_entry() == oracle.lib().orc_sizeof_entry() == 24
+    assert fpx.ENTRY_DTYPE == oracle.ENTRY_DTYPE
+    # key packing: site << 32 | fmt << 4 | flow << 2 | kind (FPX_KEY in the header)
+    src = open(HEADER).read()
+    assert "((uint64_t)(site) << 32) | ((uint64_t)(fmt) << 4) | ((uint64_t)(flow) << 2) | (uint64_t)(kind)" in src
+    assert oracle.key(7, 3, 2, 1) == (7 << 32) | (3 << 4) | (2 << 2) | 1
+
+
+def test_calls_without_device_fail_cleanly():
+    from paper_conf_hpdc_lilfslg23_b200 import fpx
+
+    h = ctypes.c_void_p()
+    st = fpx.lib.fpx_open(0, None, ctypes.byref(h))
+    assert st in (fpx.ERR_CUDA, fpx.ERR_INVALID, fpx.OK)
+    if st == fpx.OK:  # a GPU is present: nothing to check here
+        fpx.lib.fpx_close(h)
+        return
+    assert not h.value
+    assert fpx.lib.fpx_open(0, None, None) == fpx.ERR_INVALID
+    assert fpx.lib.fpx_scan_records(None, None, 1, None, 0, 0, 0, None) == fpx.ERR_INVALID
+    assert fpx.lib.fpx_table_fetch(None, None, 0, None, 0) == fpx.ERR_INVALID
+    assert fpx.lib.fpx_close(None) == fpx.ERR_INVALID
+    assert fpx.lib.fpx_strerror(fpx.ERR_TABLE_FULL).startswith(b"exception table full")
+
+
+def test_t4_summary_counts_distinct_sites():
+    from paper_conf_hpdc_lilfslg23_b200 import fpx
+
+    e = np.zeros(5, dtype=fpx.ENTRY_DTYPE)
+    e["site"] = [1, 1, 2, 3, 3]
+    e["fmt"] = [0, 0, 0, 1, 0]
+    e["kind"] = [0, 0, 0, 2, 1]
+    e["flow"] = [0, 1, 2, 0, 0]
+    assert fpx.t4_summary(e) == {(0, 0): 2, (1, 2): 1, (0, 1): 1}
