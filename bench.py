@@ -225,6 +225,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--variant", default="tma", choices=["tma", "ldg"], help="record-scan kernel (ldg = ablation)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     cfg = dict(CONFIGS[args.config])
@@ -254,7 +255,7 @@ def main():
     lane_values, nbytes = workload_stats(hdr, cfg["mode"])
     torch.cuda.synchronize()
 
-    h = fpx.Handle(local)
+    h = fpx.Handle(local, flags=fpx.OPT_SCAN_LDG if args.variant == "ldg" else 0)
     stream = torch.cuda.current_stream(dev)
     n = cfg["n"]
 
@@ -382,7 +383,7 @@ def main():
             "unit": "GB/s",
             "frac": achieved / peak,
             "traffic": traffic,
-            "kernel": "k_scan_records",
+            "kernel": "k_scan_records_" + args.variant,
             "kernel_ms": kern_ms,
             "peak_source": peak_src,
         },

@@ -16,6 +16,7 @@ using namespace fpx;
 struct fpx_ctx {
   int device = 0;
   int num_sms = 148;
+  uint32_t variant = 0;  // record-scan kernel: 0 TMA ring, 1 LDG (ablation)
   uint64_t slots = 0;
   TableView tv{};
   uint64_t newlog_cursor = 0;  // FETCH_NEW position
@@ -159,7 +160,7 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   *out = nullptr;
   fpx_options o{};
   if (opt) o = *opt;
-  if (o.flags != 0) return FPX_ERR_INVALID;
+  if ((o.flags & ~(uint32_t)FPX_OPT_SCAN_LDG) != 0) return FPX_ERR_INVALID;
   if (o.table_log2_slots == 0) o.table_log2_slots = 20;
   if (o.table_log2_slots < 4 || o.table_log2_slots > 30) return FPX_ERR_INVALID;
   int ndev = 0;
@@ -170,6 +171,7 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   fpx_ctx* h = new (std::nothrow) fpx_ctx();
   if (!h) return FPX_ERR_NOMEM;
   h->device = device;
+  h->variant = (o.flags & FPX_OPT_SCAN_LDG) ? 1u : 0u;
   CK(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, device));
   h->slots = 1ull << o.table_log2_slots;
   // the log never holds more keys than the table has slots
@@ -209,7 +211,8 @@ fpx_status fpx_scan_records(fpx_handle h, const fpx_rec_hdr* d_hdr, uint64_t n_r
   DeviceGuard g(h->device);
   if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
-  CK(launch_scan_records(d_hdr, n_records, d_arena, arena_planes, base_index, mode, h->tv, h->num_sms, s));
+  CK(launch_scan_records(d_hdr, n_records, d_arena, arena_planes, base_index, mode, h->tv, h->num_sms, h->variant,
+                         s));
   h->last_stream = s;
   return FPX_OK;
 }

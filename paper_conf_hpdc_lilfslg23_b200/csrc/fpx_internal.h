@@ -41,10 +41,11 @@ struct TableView {
   Ctl* ctl;
 };
 
-// ---- launchers (fpx_scan.cu, fpx_table.cu) --------------------------------
+// ---- launchers (fpx_scan_records.cu, fpx_scan_tensor.cu, fpx_table.cu) --------------------------------
+// variant 0 = TMA ring (default), 1 = register-staged LDG (FPX_OPT_SCAN_LDG ablation)
 cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena,
                                 uint64_t arena_planes, uint64_t base_index, uint32_t mode,
-                                const TableView& tv, int num_sms, cudaStream_t s);
+                                const TableView& tv, int num_sms, uint32_t variant, cudaStream_t s);
 cudaError_t launch_scan_tensor(const void* d_ptr, uint64_t n_elems, uint32_t fmt, uint32_t site,
                                uint64_t base_index, const TableView& tv, int num_sms, cudaStream_t s);
 cudaError_t launch_table_reset(const TableView& tv, uint64_t slots, cudaStream_t s);

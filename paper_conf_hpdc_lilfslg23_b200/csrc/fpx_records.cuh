@@ -1,0 +1,171 @@
+// fpx_records.cuh — record decoding, validation and the exact per-record
+// evaluation shared by the record-scan kernels.
+//
+//   record_valid  the header contract of include/fpx.h
+//   eval_record   one lane of one record, exactly: Alg1's kind dispatch
+//                  on every destination value (detector) or the
+//                 Table 2 state over dest + pre-execution sources
+//                 (analyzer)
+//   exact_tile    eval_record + warp aggregation + table update for every
+//                 record of a tile (the rare path: tiles with an exception)
+//   item_counts   planes of a record the fast path must look at, per format
+#pragma once
+#include "fpx_device.cuh"
+
+namespace fpx {
+namespace rec {
+
+
+constexpr int TILE = 32;  // records per warp tile (one header per lane)
+
+struct alignas(16) RecDesc {
+  uint32_t val_off, mask, meta, site;
+};
+
+__device__ __forceinline__ uint32_t op_of(uint32_t meta) { return meta & 0xFFu; }
+__device__ __forceinline__ uint32_t fmt_of(uint32_t meta) { return (meta >> 8) & 3u; }
+__device__ __forceinline__ uint32_t nsrc_of(uint32_t meta) { return (meta >> 10) & 3u; }
+__device__ __forceinline__ uint32_t dwords_of(uint32_t meta) { return (meta >> 12) & 7u; }
+__device__ __forceinline__ uint32_t sw_of(uint32_t fmt) { return fmt == FPX_FP64 ? 2u : 1u; }
+__device__ __forceinline__ bool is_compare(uint32_t op) {
+  return op == FPX_OP_FSETP || op == FPX_OP_DSETP || op == FPX_OP_FSET;
+}
+
+// Header validation (include/fpx.h record contract).
+template <int MODE>
+__device__ __forceinline__ bool record_valid(const uint4 h, uint64_t arena_planes) {
+  const uint32_t meta = h.z, fmt = fmt_of(meta), dw = dwords_of(meta);
+  bool ok = h.x != FPX_SITE_INVALID;
+  ok &= (meta >> 15) == 0u;
+  ok &= op_of(meta) < FPX_OP_COUNT;
+  ok &= dw <= 4u;
+  ok &= !(fmt == FPX_FP64 && (dw & 1u));
+  const uint64_t planes = dw + (uint64_t)nsrc_of(meta) * sw_of(fmt);
+  ok &= (uint64_t)h.w + planes <= arena_planes;
+  if (MODE == FPX_MODE_FLOW) {
+    ok &= (fmt == FPX_FP32 || fmt == FPX_FP64);
+    ok &= (dw == 0u || dw == sw_of(fmt));
+  }
+  return ok;
+}
+
+// Sign-extended "lane is active" mask: all ones if bit `lane` of m is set.
+__device__ __forceinline__ uint32_t lane_ext(uint32_t m, int lane) {
+  return (uint32_t)((int32_t)(m << (31 - lane)) >> 31);
+}
+
+// Exact evaluation of one record for this lane (both modes).  Returns the
+// bitmask of event codes held by this lane; codes / evm describe per-value
+// codes for count_of().
+template <int MODE>
+__device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t* __restrict__ lane_base, int lane,
+                                                uint32_t& codes, uint32_t& evm) {
+  codes = 0;
+  evm = 0;
+  if (((d.mask >> lane) & 1u) == 0u) return 0u;
+  const uint32_t op = op_of(d.meta), fmt = fmt_of(d.meta), nsrc = nsrc_of(d.meta), dw = dwords_of(d.meta);
+  const uint32_t sw = sw_of(fmt);
+  const bool have_div = (op == FPX_OP_DIV) && nsrc >= 2 && dw == sw;
+  // destination words d[0..dw) and source words s[0..ns_words) of this lane
+  uint32_t ns_words = 0;
+  if (MODE == FPX_MODE_FLOW) ns_words = nsrc * sw;
+  else if (have_div) ns_words = 2 * sw;
+  const uint32_t* p = lane_base + (uint64_t)d.val_off * 32;
+  uint32_t dv[4], sv[6];
+#pragma unroll
+  for (uint32_t k = 0; k < 4; ++k) dv[k] = k < dw ? p[(uint64_t)k * 32] : 0u;
+#pragma unroll
+  for (uint32_t k = 0; k < 6; ++k) sv[k] = k < ns_words ? p[(uint64_t)(dw + k) * 32] : 0u;
+
+  if (MODE == FPX_MODE_DEST) {
+    const uint32_t nv = fmt == FPX_FP64 ? dw / 2 : fmt == FPX_FP32 ? dw : 2 * dw;
+    uint32_t cm = 0;
+#pragma unroll
+    for (uint32_t v = 0; v < 8; ++v) {
+      if (v >= nv) break;
+      uint32_t lo, hi = 0, nlo, nhi = 0, dlo, dhi = 0;  // value, dividend, divisor
+      if (fmt == FPX_FP64) {
+        lo = dv[(2 * v) & 3];
+        hi = dv[(2 * v + 1) & 3];
+        nlo = sv[0]; nhi = sv[1]; dlo = sv[2]; dhi = sv[3];
+      } else if (fmt == FPX_FP32) {
+        lo = dv[v & 3];
+        nlo = sv[0]; dlo = sv[1];
+      } else {
+        const uint32_t sh = 16u * (v & 1u);
+        lo = (dv[(v / 2) & 3] >> sh) & 0xFFFFu;
+        nlo = (sv[0] >> sh) & 0xFFFFu;
+        dlo = (sv[1] >> sh) & 0xFFFFu;
+      }
+      const int k = dest_kind(op, fmt, lo, hi, have_div, nlo, nhi, dlo, dhi);
+      if (k >= 0) {
+        codes |= (uint32_t)k << (4 * v);
+        evm |= 1u << v;
+        cm |= 1u << k;
+      }
+    }
+    return cm;
+  } else {
+    // Analyzer: S = most severe class among the pre-execution sources.
+    int S = CODE_NONE, sev = 0;
+#pragma unroll
+    for (uint32_t k = 0; k < 3; ++k) {
+      if (k >= nsrc) break;
+      const uint32_t c = fmt == FPX_FP64 ? cls_fp64(sv[2 * k], sv[2 * k + 1]) : cls_fp32(sv[k]);
+      const int sv_ = c == CLS_NAN ? 3 : c == CLS_INF ? 2 : c == CLS_SUB ? 1 : 0;
+      if (sv_ > sev) { sev = sv_; S = kind_of_cls(c); }
+    }
+    int D = CODE_NONE;
+    if (dw != 0u) {
+      if (fmt == FPX_FP64) D = dest_kind(op, fmt, dv[0], dv[1], have_div, sv[0], sv[1], sv[2], sv[3]);
+      else D = dest_kind(op, fmt, dv[0], 0u, have_div, sv[0], 0u, sv[1], 0u);
+    }
+    int code = CODE_NONE;
+    if (D >= 0 && S < 0) code = (FPX_GEN << 2) | D;
+    else if (D >= 0) code = (FPX_PROP << 2) | D;
+    else if (S >= 0) code = (FPX_KILL << 2) | S;
+    if (code < 0) return 0u;
+    codes = (uint32_t)code;
+    evm = 1u;
+    return 1u << code;
+  }
+}
+
+template <int MODE>
+__device__ __noinline__ void exact_tile(const RecDesc* __restrict__ recs, const uint32_t* __restrict__ lane_base,
+                                        int lane, uint64_t gidx0, const TableView tv) {
+  for (int j = 0; j < TILE; ++j) {
+    const RecDesc d = recs[j];
+    if (d.mask == 0u) continue;  // warp-uniform
+    if (MODE == FPX_MODE_DEST && is_compare(op_of(d.meta))) continue;
+    uint32_t codes, evm;
+    const uint32_t cm = eval_record<MODE>(d, lane_base, lane, codes, evm);
+    warp_flush(tv, cm, d.site, fmt_of(d.meta), gidx0 + j, [&](int c) {
+      uint32_t n = 0;
+#pragma unroll
+      for (int v = 0; v < 8; ++v) n += (((evm >> v) & 1u) && (((codes >> (4 * v)) & 15u) == (uint32_t)c)) ? 1u : 0u;
+      return n;
+    });
+  }
+}
+
+// Plane items of one record for the fast path, by list:
+//   0: FP32 words, 1: FP64 (lo, hi) pairs, 2: FP16x2 words, 3: BF16x2 words.
+template <int MODE>
+__device__ __forceinline__ uint32_t item_counts(uint32_t meta, bool ok, bool& force) {
+  force = false;
+  if (!ok) return 0u;
+  const uint32_t op = op_of(meta), fmt = fmt_of(meta), dw = dwords_of(meta), ns = nsrc_of(meta);
+  if (op == FPX_OP_DIV) { force = true; return 0u; }  // DIV0 needs the sources: exact path
+  uint32_t n;
+  if (MODE == FPX_MODE_DEST) {
+    if (is_compare(op)) return 0u;
+    n = fmt == FPX_FP64 ? dw / 2 : dw;
+  } else {
+    n = fmt == FPX_FP64 ? (dw + 2 * ns) / 2 : dw + ns;
+  }
+  return n << (8 * fmt);
+}
+
+}  // namespace rec
+}  // namespace fpx

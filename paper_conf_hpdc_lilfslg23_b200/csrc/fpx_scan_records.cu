@@ -1,0 +1,456 @@
+// fpx_scan_records.cu — the record scan for sm_100a.
+//
+// One warp owns a contiguous range of records and walks it in tiles of up to
+// 32 records (one header per lane) whose needed planes fit one stage of a
+// per-warp shared-memory ring.  Lane l of the scanning warp reads lane l of
+// every plane: exactly the lane of the instrumented warp whose register it
+// holds (Alg2, "each thread checks its own value").
+//
+// k_scan_records_tma (default)
+//   produce   lane j decodes + validates header j (prefetched one tile ahead),
+//             a warp scan assigns each record's needed planes (DEST: the
+//             destination words; FLOW: destination + sources) a contiguous
+//             slot range in the stage; runs of records whose planes are
+//             adjacent in the arena become ONE cp.async.bulk (TMA) copy
+//             global -> shared, completing on the stage's mbarrier.  Tiles
+//             are issued STAGES-1 ahead, so memory parallelism is bounded by
+//             shared memory, not registers.
+//   consume   per plane one conflict-free 32-bit LDS per lane; a few integer
+//             ops per value keep min / max witnesses of "subnormal" and
+//             "exponent all ones"; one vote per tile (the common case at 1e-6
+//             density is "nothing exceptional")
+//   exact     hit tiles only: rec::exact_tile (kind rule, flow states, warp
+//             aggregation, table) — fpx_records.cuh
+//
+// k_scan_records_ldg (ablation, FPX_OPT_SCAN_LDG): the same fast path with
+// register-staged LDG loads, batched U per warp; kept to show what the TMA
+// ring buys (profiles/).
+#include <cuda_runtime.h>
+
+#include "fpx_records.cuh"
+
+namespace fpx {
+namespace {
+
+using namespace rec;
+
+// ---- PTX wrappers: mbarrier + bulk async copy -------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_init_fence() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  while (!mbar_try_wait(bar, parity)) {
+  }
+}
+// global -> shared bulk copy (TMA), completion counted in bytes on `bar`;
+// streaming data: evict-first in L2.
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy)
+      : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// ---- TMA-ring kernel ------------------------------------------------------------
+constexpr int TMA_WARPS = 8;   // warps per CTA (one CTA per SM)
+constexpr int STAGES = 3;      // ring depth per warp (STAGES-1 tiles in flight)
+constexpr int PLANES = 64;     // planes per stage (8 KB)
+
+struct StageMeta {
+  uint32_t k;                    // records in the tile (0 = no tile)
+  uint32_t n32, n64, n16, nb16;  // fast-path items per list
+  uint32_t force;                // tile holds a record that must take the exact path
+  uint64_t gidx0;                // global index of the tile's first record
+};
+
+struct WarpSmem {
+  uint32_t planes[STAGES][PLANES * 32];  // 128 B per plane
+  uint2 items[STAGES][PLANES];           // {slot, active mask}
+  RecDesc recs[STAGES][TILE];
+  StageMeta meta[STAGES];
+  uint64_t bar[STAGES];
+};
+constexpr size_t TMA_SMEM = sizeof(WarpSmem) * TMA_WARPS;
+static_assert(TMA_SMEM <= 227 * 1024, "ring exceeds shared memory");
+
+// Planes of a valid, active record the mode must look at (all contiguous from
+// plane 0 of the record).
+template <int MODE>
+__device__ __forceinline__ uint32_t needed_planes(uint32_t meta) {
+  const uint32_t op = op_of(meta), fmt = fmt_of(meta), dw = dwords_of(meta), ns = nsrc_of(meta);
+  if (op == FPX_OP_DIV) return 0u;  // exact path reads DIV records itself
+  if (MODE == FPX_MODE_DEST) return is_compare(op) ? 0u : dw;
+  return dw + ns * sw_of(fmt);
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(TMA_WARPS * 32, 1)
+k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __restrict__ arena,
+                   uint64_t arena_planes, uint64_t base_index, uint64_t recs_per_warp, const TableView tv) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  WarpSmem& sm = reinterpret_cast<WarpSmem*>(smem_raw)[warp];
+  const uint64_t gw = blockIdx.x * (uint64_t)TMA_WARPS + warp;
+  const uint64_t start = gw * recs_per_warp;
+  if (start >= n) return;  // warp-uniform; no block-wide barriers below
+  const uint64_t end = min(n, start + recs_per_warp);
+  const uint32_t* __restrict__ lane_base = arena + lane;
+  const uint64_t policy = policy_evict_first();
+
+  if (lane == 0) {
+#pragma unroll
+    for (int s = 0; s < STAGES; ++s) mbar_init(&sm.bar[s], 1);
+    mbar_init_fence();
+  }
+  __syncwarp();
+
+  uint64_t cursor = start;
+  uint4 h = make_uint4(0, 0, 0, 0);
+  if (cursor + lane < end) h = ld_stream4(hdr + cursor + lane);
+
+  // Build tile `s` from the prefetched headers and issue its copies.
+  auto produce = [&](int s) {
+    StageMeta& m = sm.meta[s];
+    if (cursor >= end) {
+      __syncwarp();
+      if (lane == 0) m.k = 0;
+      __syncwarp();
+      return;
+    }
+    const bool inrange = cursor + lane < end;
+    const bool ok = inrange && record_valid<MODE>(h, arena_planes);
+    const uint32_t mask = ok ? h.y : 0u;
+    const uint32_t c = (ok && mask != 0u) ? needed_planes<MODE>(h.z) : 0u;
+    uint32_t incl = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(FULL, incl, o);
+      if (lane >= o) incl += t;
+    }
+    // the tile = leading records whose planes fit the stage (>= 1 record)
+    const uint32_t k = __popc(__ballot_sync(FULL, inrange && incl <= (uint32_t)PLANES));
+    const bool in_tile = (uint32_t)lane < k;
+    const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
+    if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
+    const uint32_t cc = in_tile ? c : 0u;
+    const uint32_t slot = incl - c;
+    const uint32_t total = __shfl_sync(FULL, incl, k - 1);
+    bool force = false;
+    const uint32_t cnt = item_counts<MODE>(h.z, in_tile && ok && mask != 0u, force);
+
+    // items: exclusive scan of the packed per-format counts
+    uint32_t ic = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(FULL, ic, o);
+      if (lane >= o) ic += t;
+    }
+    const uint32_t itot = __shfl_sync(FULL, ic, 31);
+    const uint32_t iex = ic - cnt;
+    const uint32_t n32 = itot & 0xFFu, n64 = (itot >> 8) & 0xFFu, n16 = (itot >> 16) & 0xFFu, nb16 = itot >> 24;
+    // the ring slot may still be read by the previous consume of this stage:
+    // order those generic reads before the async-proxy writes below
+    __syncwarp();
+    fence_proxy_async_smem();
+    sm.recs[s][lane] = in_tile ? RecDesc{h.w, mask, h.z, h.x} : RecDesc{0u, 0u, 0u, 0u};
+    if (cnt != 0u) {
+      const uint32_t fmt = fmt_of(h.z);
+      const uint32_t my = (cnt >> (8 * fmt)) & 0xFFu;
+      const uint32_t seg = fmt == 0u ? 0u : fmt == 1u ? n32 : fmt == 2u ? n32 + n64 : n32 + n64 + n16;
+      const uint32_t at = seg + ((iex >> (8 * fmt)) & 0xFFu);
+      const uint32_t step = fmt == FPX_FP64 ? 2u : 1u;
+      for (uint32_t q = 0; q < my; ++q) sm.items[s][at + q] = make_uint2(slot + q * step, mask);
+    }
+    const bool force_any = __any_sync(FULL, force);
+    if (lane == 0) {
+      m.k = k;
+      m.n32 = n32;
+      m.n64 = n64;
+      m.n16 = n16;
+      m.nb16 = nb16;
+      m.force = force_any ? 1u : 0u;
+      m.gidx0 = base_index + cursor;
+    }
+    // runs of arena-adjacent records -> one bulk copy each
+    const uint32_t a = h.w;
+    const uint32_t prev_end = __shfl_up_sync(FULL, a + cc, 1);
+    const uint32_t prev_c = __shfl_up_sync(FULL, cc, 1);
+    const bool head = cc != 0u && (lane == 0 || prev_c == 0u || prev_end != a);
+    const uint32_t heads = __ballot_sync(FULL, head);
+    const uint32_t above = lane == 31 ? 0u : heads & (0xFFFFFFFFu << (lane + 1));  // heads above this lane
+    const uint32_t next = above ? (uint32_t)(__ffs(above) - 1) : 32u;
+    const uint32_t next_slot_raw = __shfl_sync(FULL, slot, next & 31u);
+    const uint32_t run_end = next < k ? next_slot_raw : total;
+    __syncwarp();
+    if (lane == 0) mbar_arrive_expect_tx(&sm.bar[s], total * 128u);
+    __syncwarp();
+    if (head) bulk_g2s(&sm.planes[s][slot * 32], arena + (uint64_t)a * 32, (run_end - slot) * 128u, &sm.bar[s], policy);
+    // advance and prefetch the next tile's headers
+    cursor += k;
+    h = make_uint4(0, 0, 0, 0);
+    if (cursor + lane < end) h = ld_stream4(hdr + cursor + lane);
+  };
+
+  uint32_t phase = 0;  // bit s = parity to wait for on stage s
+#pragma unroll 1
+  for (int s = 0; s < STAGES - 1; ++s) produce(s);
+#pragma unroll 1
+  for (uint32_t i = 0;; ++i) {
+    const int s = (int)(i % STAGES);
+    produce((int)((i + STAGES - 1) % STAGES));
+    const StageMeta m = sm.meta[s];
+    if (m.k == 0u) break;
+    mbar_wait(&sm.bar[s], (phase >> s) & 1u);
+    phase ^= 1u << s;
+
+    // ---- fast path over the staged planes --------------------------------
+    const uint32_t* __restrict__ pl = sm.planes[s];
+    const uint2* __restrict__ it = sm.items[s];
+    uint32_t mn32 = 0xFFFFFFFFu, mx32 = 0u, mn64 = 0xFFFFFFFFu, mx64 = 0u;
+    uint32_t mn16 = 0xFFFFFFFFu, mx16 = 0u, mnb = 0xFFFFFFFFu, mxb = 0u;
+#pragma unroll 4
+    for (uint32_t q = 0; q < m.n32; ++q) {
+      const uint2 t = it[q];
+      const uint32_t x = pl[t.x * 32 + lane] & 0x7FFFFFFFu & lane_ext(t.y, lane);
+      mn32 = min(mn32, x - 1u);  // < 0x7FFFFF  <=> subnormal
+      mx32 = max(mx32, x);       // > 0x7F7FFFFF <=> INF / NaN
+    }
+#pragma unroll 4
+    for (uint32_t q = 0; q < m.n64; ++q) {
+      const uint2 t = it[m.n32 + q];
+      const uint32_t e = lane_ext(t.y, lane);
+      const uint32_t lo = pl[t.x * 32 + lane] & e;
+      const uint32_t ah = pl[(t.x + 1) * 32 + lane] & 0x7FFFFFFFu & e;
+      const uint32_t a2 = (ah << 1) | min(lo, 1u);  // 0 zero, [1,0x1FFFFF] SUB, >= 0xFFE00000 INF/NaN
+      mn64 = min(mn64, a2 - 1u);
+      mx64 = max(mx64, a2);
+    }
+#pragma unroll 4
+    for (uint32_t q = 0; q < m.n16 + m.nb16; ++q) {
+      const uint2 t = it[m.n32 + m.n64 + q];
+      const uint32_t x = pl[t.x * 32 + lane] & 0x7FFF7FFFu & lane_ext(t.y, lane);
+      const uint32_t l = x & 0xFFFFu, hh = x >> 16;
+      if (q < m.n16) {
+        mn16 = min(mn16, min(l - 1u, hh - 1u));
+        mx16 = max(mx16, max(l, hh));
+      } else {
+        mnb = min(mnb, min(l - 1u, hh - 1u));
+        mxb = max(mxb, max(l, hh));
+      }
+    }
+    const bool hit = mn32 < 0x007FFFFFu || mx32 > 0x7F7FFFFFu || mn64 < 0x001FFFFFu || mx64 >= 0xFFE00000u ||
+                     mn16 < 0x03FFu || mx16 > 0x7BFFu || mnb < 0x007Fu || mxb > 0x7F7Fu;
+    if (__any_sync(FULL, hit) || m.force) exact_tile<MODE>(sm.recs[s], lane_base, lane, m.gidx0, tv);
+  }
+}
+
+// ---- register-staged LDG kernel (ablation) ------------------------------------
+constexpr int LDG_WARPS = 8;
+constexpr int MAXITEMS = 128;  // <= 4 items per record
+constexpr int U32 = 8;         // FP32 / packed items per load batch
+constexpr int U64 = 4;         // FP64 pairs per load batch
+
+template <int MODE>
+__global__ void __launch_bounds__(LDG_WARPS * 32, 4)
+k_scan_records_ldg(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __restrict__ arena,
+               uint64_t arena_planes, uint64_t base_index, const TableView tv) {
+  __shared__ RecDesc s_rec[LDG_WARPS][TILE];
+  __shared__ uint2 s_item[LDG_WARPS][MAXITEMS];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint64_t nwarps = (uint64_t)gridDim.x * LDG_WARPS;
+  const uint64_t ntiles = (n + TILE - 1) / TILE;
+  const uint32_t* __restrict__ lane_base = arena + lane;
+  RecDesc* __restrict__ recs = s_rec[warp];
+  uint2* __restrict__ items = s_item[warp];
+
+  uint64_t tile = blockIdx.x * (uint64_t)LDG_WARPS + warp;
+  uint4 h_next = make_uint4(0, 0, 0, 0);
+  if (tile < ntiles && tile * TILE + lane < n) h_next = ld_stream4(hdr + tile * TILE + lane);
+
+  for (; tile < ntiles; tile += nwarps) {
+    // ---- prologue: lane = record --------------------------------------------
+    const uint64_t r = tile * TILE + lane;
+    const bool inrange = r < n;
+    const uint4 h = h_next;
+    {
+      const uint64_t nt = tile + nwarps;  // prefetch the next tile's header
+      if (nt < ntiles && nt * TILE + lane < n) h_next = ld_stream4(hdr + nt * TILE + lane);
+    }
+    const bool ok = inrange && record_valid<MODE>(h, arena_planes);
+    const uint32_t bad = __ballot_sync(FULL, inrange && !ok);
+    if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
+    const uint32_t mask = ok ? h.y : 0u;
+    bool force;
+    const uint32_t cnt = item_counts<MODE>(h.z, ok && mask != 0u, force);
+    __syncwarp();
+    recs[lane] = RecDesc{h.w, mask, h.z, h.x};
+    // exclusive scan of the four packed 8-bit counts (sums stay <= 128)
+    uint32_t incl = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(FULL, incl, o);
+      if (lane >= o) incl += t;
+    }
+    const uint32_t tot = __shfl_sync(FULL, incl, 31);
+    const uint32_t excl = incl - cnt;
+    const uint32_t n32 = tot & 0xFFu, n64 = (tot >> 8) & 0xFFu, n16 = (tot >> 16) & 0xFFu, nb16 = tot >> 24;
+    if (cnt != 0u) {
+      const uint32_t fmt = fmt_of(h.z);
+      const uint32_t my = (cnt >> (8 * fmt)) & 0xFFu;
+      const uint32_t seg = fmt == 0u ? 0u : fmt == 1u ? n32 : fmt == 2u ? n32 + n64 : n32 + n64 + n16;
+      const uint32_t at = seg + ((excl >> (8 * fmt)) & 0xFFu);
+      const uint32_t step = fmt == FPX_FP64 ? 2u : 1u;
+      for (uint32_t k = 0; k < my; ++k) items[at + k] = make_uint2(h.w + k * step, mask);
+    }
+    const bool force_any = __any_sync(FULL, force);
+    __syncwarp();
+
+    // ---- fast path: min / max witnesses per format ---------------------------
+    uint32_t mn32 = 0xFFFFFFFFu, mx32 = 0u, mn64 = 0xFFFFFFFFu, mx64 = 0u;
+    uint32_t mn16 = 0xFFFFFFFFu, mx16 = 0u, mnb = 0xFFFFFFFFu, mxb = 0u;
+    for (uint32_t i = 0; i < n32; i += U32) {
+      uint32_t w[U32], m[U32];
+#pragma unroll
+      for (int u = 0; u < U32; ++u) {
+        m[u] = 0u;
+        w[u] = 0u;
+        if (i + u < n32) {
+          const uint2 it = items[i + u];
+          m[u] = it.y;
+          w[u] = ld_stream(lane_base + (uint64_t)it.x * 32);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < U32; ++u) {
+        const uint32_t a = w[u] & 0x7FFFFFFFu & lane_ext(m[u], lane);
+        mn32 = min(mn32, a - 1u);  // < 0x7FFFFF  <=> subnormal
+        mx32 = max(mx32, a);       // > 0x7F7FFFFF <=> INF / NaN
+      }
+    }
+    for (uint32_t i = 0; i < n64; i += U64) {
+      uint32_t lo[U64], hi[U64], m[U64];
+#pragma unroll
+      for (int u = 0; u < U64; ++u) {
+        m[u] = 0u;
+        lo[u] = 0u;
+        hi[u] = 0u;
+        if (i + u < n64) {
+          const uint2 it = items[n32 + i + u];
+          m[u] = it.y;
+          const uint32_t* p = lane_base + (uint64_t)it.x * 32;
+          lo[u] = ld_stream(p);
+          hi[u] = ld_stream(p + 32);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < U64; ++u) {
+        const uint32_t e = lane_ext(m[u], lane);
+        const uint32_t ah = hi[u] & 0x7FFFFFFFu & e;
+        const uint32_t a2 = (ah << 1) | min(lo[u] & e, 1u);  // 0 zero, [1,0x1FFFFF] SUB, >=0xFFE00000 INF/NaN
+        mn64 = min(mn64, a2 - 1u);
+        mx64 = max(mx64, a2);
+      }
+    }
+    for (uint32_t i = 0; i < n16 + nb16; i += U32) {
+      uint32_t w[U32], m[U32];
+#pragma unroll
+      for (int u = 0; u < U32; ++u) {
+        m[u] = 0u;
+        w[u] = 0u;
+        if (i + u < n16 + nb16) {
+          const uint2 it = items[n32 + n64 + i + u];
+          m[u] = it.y;
+          w[u] = ld_stream(lane_base + (uint64_t)it.x * 32);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < U32; ++u) {
+        const uint32_t x = w[u] & 0x7FFF7FFFu & lane_ext(m[u], lane);
+        const uint32_t l = x & 0xFFFFu, hh = x >> 16;
+        if (i + u < n16) {
+          mn16 = min(mn16, min(l - 1u, hh - 1u));
+          mx16 = max(mx16, max(l, hh));
+        } else {
+          mnb = min(mnb, min(l - 1u, hh - 1u));
+          mxb = max(mxb, max(l, hh));
+        }
+      }
+    }
+    const bool hit = mn32 < 0x007FFFFFu || mx32 > 0x7F7FFFFFu || mn64 < 0x001FFFFFu || mx64 >= 0xFFE00000u ||
+                     mn16 < 0x03FFu || mx16 > 0x7BFFu || mnb < 0x007Fu || mxb > 0x7F7Fu;
+    if (__any_sync(FULL, hit) || force_any) exact_tile<MODE>(recs, lane_base, lane, base_index + tile * TILE, tv);
+  }
+}
+
+
+template <int MODE>
+cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena, uint64_t arena_planes,
+                             uint64_t base_index, const TableView& tv, int num_sms, uint32_t variant,
+                             cudaStream_t s) {
+  if (variant == 1u) {
+    const uint64_t tiles = (n + TILE - 1) / TILE;
+    uint64_t blocks = (tiles + LDG_WARPS - 1) / LDG_WARPS;
+    const uint64_t cap = (uint64_t)num_sms * 4;
+    if (blocks > cap) blocks = cap;
+    k_scan_records_ldg<MODE><<<(unsigned)blocks, LDG_WARPS * 32, 0, s>>>(reinterpret_cast<const uint4*>(d_hdr), n,
+                                                                         d_arena, arena_planes, base_index, tv);
+    return cudaGetLastError();
+  }
+  static bool attr_set[64] = {};  // per device
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 64 || !attr_set[dev]) {
+    cudaError_t e = cudaFuncSetAttribute(k_scan_records_tma<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)TMA_SMEM);
+    if (e != cudaSuccess) return e;
+    if (dev < 64) attr_set[dev] = true;
+  }
+  // one CTA per SM; each warp a contiguous range of records (whole tiles of 32
+  // where possible, so that ranges stay 512-B aligned in the header array)
+  const uint64_t warps = (uint64_t)num_sms * TMA_WARPS;
+  uint64_t per = (n + warps - 1) / warps;
+  per = (per + TILE - 1) / TILE * TILE;
+  const uint64_t blocks = ((n + per - 1) / per + TMA_WARPS - 1) / TMA_WARPS;
+  k_scan_records_tma<MODE><<<(unsigned)blocks, TMA_WARPS * 32, TMA_SMEM, s>>>(
+      reinterpret_cast<const uint4*>(d_hdr), n, d_arena, arena_planes, base_index, per, tv);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena, uint64_t arena_planes,
+                                uint64_t base_index, uint32_t mode, const TableView& tv, int num_sms, uint32_t variant,
+                                cudaStream_t s) {
+  if (mode == FPX_MODE_DEST)
+    return launch_records_t<FPX_MODE_DEST>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, s);
+  return launch_records_t<FPX_MODE_FLOW>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, s);
+}
+
+}  // namespace fpx

@@ -1,0 +1,208 @@
+// fpx_scan_tensor.cu — destination-only scan of a plain FP32/FP64/FP16/BF16
+// buffer (the SRU case P:711-715 recast for model activations).
+//
+// 128-bit loads of the 16-B-aligned body, TU vectors in flight per thread,
+// grid-stride over a persistent grid (8 CTAs x 256 threads per SM).  A few
+// integer ops per value keep min / max witnesses of "subnormal" and
+// "exponent all ones"; one vote per batch; exact classification, per-kind
+// warp reduction and table update only for hit batches.  Misaligned heads and
+// ragged tails (< one vector each) are classified by one warp.
+#include <cuda_runtime.h>
+
+#include "fpx_device.cuh"
+
+namespace fpx {
+namespace {
+
+template <uint32_t FMT>
+struct TensorTraits;
+template <>
+struct TensorTraits<FPX_FP32> {
+  static constexpr uint32_t V = 4;  // values per 16 B
+};
+template <>
+struct TensorTraits<FPX_FP64> {
+  static constexpr uint32_t V = 2;
+};
+template <>
+struct TensorTraits<FPX_FP16> {
+  static constexpr uint32_t V = 8;
+};
+template <>
+struct TensorTraits<FPX_BF16> {
+  static constexpr uint32_t V = 8;
+};
+
+// class of value e (0..V-1) of a 16-B vector
+template <uint32_t FMT>
+__device__ __forceinline__ uint32_t vec_cls(const uint4& q, uint32_t e) {
+  const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+  if (FMT == FPX_FP32) return cls_fp32(w[e]);
+  if (FMT == FPX_FP64) return cls_fp64(w[2 * e], w[2 * e + 1]);
+  const uint32_t half = (w[e / 2] >> (16 * (e & 1))) & 0xFFFFu;
+  return FMT == FPX_FP16 ? cls_fp16(half) : cls_bf16(half);
+}
+
+// Cheap "anything exceptional in this vector" witness update.
+template <uint32_t FMT>
+__device__ __forceinline__ void vec_witness(const uint4& q, uint32_t& mn, uint32_t& mx) {
+  if (FMT == FPX_FP32) {
+    const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const uint32_t a = w[k] & 0x7FFFFFFFu;
+      mn = min(mn, a - 1u);
+      mx = max(mx, a);
+    }
+  } else if (FMT == FPX_FP64) {
+    const uint32_t lo[2] = {q.x, q.z}, hi[2] = {q.y, q.w};
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+      const uint32_t a2 = ((hi[k] & 0x7FFFFFFFu) << 1) | min(lo[k], 1u);
+      mn = min(mn, a2 - 1u);
+      mx = max(mx, a2);
+    }
+  } else {
+    const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const uint32_t x = w[k] & 0x7FFF7FFFu;
+      const uint32_t l = x & 0xFFFFu, h = x >> 16;
+      mn = min(mn, min(l - 1u, h - 1u));
+      mx = max(mx, max(l, h));
+    }
+  }
+}
+template <uint32_t FMT>
+__device__ __forceinline__ bool witness_hit(uint32_t mn, uint32_t mx) {
+  if (FMT == FPX_FP32) return mn < 0x007FFFFFu || mx > 0x7F7FFFFFu;
+  if (FMT == FPX_FP64) return mn < 0x001FFFFFu || mx >= 0xFFE00000u;
+  if (FMT == FPX_FP16) return mn < 0x03FFu || mx > 0x7BFFu;
+  return mn < 0x007Fu || mx > 0x7F7Fu;
+}
+
+constexpr int TU = 4;  // vectors per thread per batch
+
+// Exact per-warp reduction of per-lane kind counts and first offsets.
+__device__ __forceinline__ void flush_kinds(const TableView& tv, uint32_t site, uint32_t fmt, const uint32_t cnt[3],
+                                            const uint32_t first_off[3], uint64_t idx0) {
+#pragma unroll
+  for (int k = 0; k < 3; ++k) {
+    const uint32_t tot = __reduce_add_sync(FULL, cnt[k]);
+    if (tot) {
+      const uint32_t f = __reduce_min_sync(FULL, first_off[k]);
+      if ((threadIdx.x & 31) == 0) table_add(tv, make_key(site, fmt, (uint32_t)k), tot, idx0 + f);
+    }
+  }
+}
+
+static_assert(TU == 4, "tensor_exact takes four vectors");
+
+// Exact classification of one hit batch (rare): offsets relative to the
+// warp's lowest vector of the batch, reduced per warp.
+template <uint32_t FMT>
+__device__ __noinline__ void tensor_exact(uint4 q0, uint4 q1, uint4 q2, uint4 q3, uint64_t v0, uint64_t nthr,
+                                          uint64_t nvec, int lane, uint64_t idx_base, uint32_t site,
+                                          const TableView tv) {
+  constexpr uint32_t V = TensorTraits<FMT>::V;
+  const uint4 q[TU] = {q0, q1, q2, q3};
+  const uint64_t wv0 = v0 - (uint64_t)lane;
+  uint32_t cnt[3] = {0, 0, 0}, fo[3] = {0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu};
+#pragma unroll
+  for (int u = 0; u < TU; ++u) {
+    const uint64_t v = v0 + (uint64_t)u * nthr;
+    if (v >= nvec) continue;
+#pragma unroll
+    for (uint32_t e = 0; e < V; ++e) {
+      const int k = kind_of_cls(vec_cls<FMT>(q[u], e));
+      const uint32_t off = (uint32_t)((v - wv0) * V + e);
+#pragma unroll
+      for (int kk = 0; kk < 3; ++kk)
+        if (k == kk) { cnt[kk]++; fo[kk] = min(fo[kk], off); }
+    }
+  }
+  flush_kinds(tv, site, FMT, cnt, fo, idx_base + wv0 * V);
+}
+
+template <uint32_t FMT>
+__global__ void __launch_bounds__(256, 8)
+k_scan_tensor(const uint4* __restrict__ body, uint64_t nvec, const uint8_t* __restrict__ scalars_lo,
+              uint32_t n_head, const uint8_t* __restrict__ scalars_hi, uint32_t n_tail, uint64_t idx_body,
+              uint64_t idx_tail, uint64_t base_index, uint32_t site, const TableView tv) {
+  constexpr uint32_t V = TensorTraits<FMT>::V;
+  constexpr uint32_t ES = 16 / V;
+  const int lane = threadIdx.x & 31;
+  const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+
+  // head / tail scalars (< one vector each): first warp of block 0, exact.
+  if (blockIdx.x == 0 && threadIdx.x < 32) {
+    auto one = [&](const uint8_t* q, uint32_t off, uint32_t cnt[3], uint32_t fo[3]) {
+      uint32_t lo = 0, hi = 0;
+      if (ES == 8) { lo = *(const uint32_t*)q; hi = *(const uint32_t*)(q + 4); }
+      else if (ES == 4) lo = *(const uint32_t*)q;
+      else lo = *(const uint16_t*)q;
+      const int k = kind_of_cls(cls_val(FMT, lo, hi));
+#pragma unroll
+      for (int kk = 0; kk < 3; ++kk)
+        if (k == kk) { cnt[kk]++; fo[kk] = min(fo[kk], off); }
+    };
+    uint32_t ch[3] = {0, 0, 0}, fh[3] = {0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu};
+    if ((uint32_t)lane < n_head) one(scalars_lo + (uint64_t)lane * ES, (uint32_t)lane, ch, fh);
+    flush_kinds(tv, site, FMT, ch, fh, base_index);
+    uint32_t ct[3] = {0, 0, 0}, ft[3] = {0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu};
+    if ((uint32_t)lane < n_tail) one(scalars_hi + (uint64_t)lane * ES, (uint32_t)lane, ct, ft);
+    flush_kinds(tv, site, FMT, ct, ft, base_index + idx_tail);
+  }
+
+  // body: batches of TU vectors per thread, grid-stride
+  for (uint64_t v0 = tid; v0 < nvec; v0 += nthr * TU) {
+    uint4 q[TU];
+#pragma unroll
+    for (int u = 0; u < TU; ++u) {
+      const uint64_t v = v0 + (uint64_t)u * nthr;
+      q[u] = v < nvec ? ld_stream4(body + v) : make_uint4(0, 0, 0, 0);
+    }
+    uint32_t mn = 0xFFFFFFFFu, mx = 0u;
+#pragma unroll
+    for (int u = 0; u < TU; ++u) vec_witness<FMT>(q[u], mn, mx);
+    if (__any_sync(FULL, witness_hit<FMT>(mn, mx)))
+      tensor_exact<FMT>(q[0], q[1], q[2], q[3], v0, nthr, nvec, lane, base_index + idx_body, site, tv);
+  }
+}
+
+template <uint32_t FMT>
+cudaError_t launch_tensor_t(const void* d_ptr, uint64_t n, uint32_t site, uint64_t base_index, const TableView& tv,
+                            int num_sms, cudaStream_t s) {
+  constexpr uint32_t V = TensorTraits<FMT>::V;
+  constexpr uint32_t ES = 16 / V;
+  const uintptr_t a = reinterpret_cast<uintptr_t>(d_ptr);
+  uint64_t head = ((16u - (uint32_t)(a & 15u)) & 15u) / ES;
+  if (head > n) head = n;
+  const uint64_t nvec = (n - head) / V;
+  const uint64_t tail = n - head - nvec * V;
+  const uint8_t* p = static_cast<const uint8_t*>(d_ptr);
+  const uint4* body = reinterpret_cast<const uint4*>(p + head * ES);
+  const uint8_t* tailp = p + (head + nvec * V) * ES;
+  uint64_t blocks = (nvec + 256 * TU - 1) / (256 * TU);
+  const uint64_t cap = (uint64_t)num_sms * 8;
+  if (blocks > cap) blocks = cap;
+  if (blocks == 0) blocks = 1;
+  k_scan_tensor<FMT><<<(unsigned)blocks, 256, 0, s>>>(body, nvec, p, (uint32_t)head, tailp, (uint32_t)tail, head,
+                                                       head + nvec * V, base_index, site, tv);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_scan_tensor(const void* d_ptr, uint64_t n, uint32_t fmt, uint32_t site, uint64_t base_index,
+                               const TableView& tv, int num_sms, cudaStream_t s) {
+  switch (fmt) {
+    case FPX_FP32: return launch_tensor_t<FPX_FP32>(d_ptr, n, site, base_index, tv, num_sms, s);
+    case FPX_FP64: return launch_tensor_t<FPX_FP64>(d_ptr, n, site, base_index, tv, num_sms, s);
+    case FPX_FP16: return launch_tensor_t<FPX_FP16>(d_ptr, n, site, base_index, tv, num_sms, s);
+    default: return launch_tensor_t<FPX_BF16>(d_ptr, n, site, base_index, tv, num_sms, s);
+  }
+}
+
+}  // namespace fpx

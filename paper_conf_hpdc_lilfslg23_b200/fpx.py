@@ -27,6 +27,7 @@ NAN, INF, SUB, DIV0 = 0, 1, 2, 3
 FLOW_NONE, GEN, PROP, KILL = 0, 1, 2, 3
 MODE_DEST, MODE_FLOW = 0, 1
 FETCH_ALL, FETCH_NEW = 0, 1
+OPT_SCAN_LDG = 1
 KEY_EMPTY = 0xFFFFFFFFFFFFFFFF
 
 ENTRY_DTYPE = np.dtype(
@@ -100,9 +101,9 @@ def _stream_ptr(stream) -> int:
 class Handle:
     """One fpx context on one device (fpx_open ... fpx_close)."""
 
-    def __init__(self, device: int = 0, table_log2_slots: int = 0, newlog_capacity: int = 0):
+    def __init__(self, device: int = 0, table_log2_slots: int = 0, newlog_capacity: int = 0, flags: int = 0):
         self._h = _vp()
-        opt = Options(table_log2_slots, newlog_capacity, 0)
+        opt = Options(table_log2_slots, newlog_capacity, flags)
         check(lib.fpx_open(device, ctypes.byref(opt), ctypes.byref(self._h)), "fpx_open")
         self.device = device
         self.last_status = OK

@@ -99,10 +99,11 @@ def _brute_trace():
     return tr.arrays()
 
 
+@pytest.mark.parametrize("variant", [0, 1], ids=["tma", "ldg"])
 @pytest.mark.parametrize("mode", [DEST, FLOW])
-def test_bruteforce_ieee_ops_gpu(fpx, mode):
+def test_bruteforce_ieee_ops_gpu(fpx, mode, variant):
     hdr, arena = _brute_trace()
-    got, st, _ = gpu_scan(fpx, hdr, arena, base=0, mode=mode)
+    got, st, _ = gpu_scan(fpx, hdr, arena, base=0, mode=mode, flags=variant)
     assert_same(got, oracle_scan(hdr, arena, 0, mode).entries())
 
 
@@ -116,14 +117,15 @@ RECIPES = [
 ]
 
 
+@pytest.mark.parametrize("variant", [0, 1], ids=["tma", "ldg"])
 @pytest.mark.parametrize("name,recipe,mode,n,sites", RECIPES, ids=[r[0] for r in RECIPES])
-def test_synthetic_trace_parity(fpx, name, recipe, mode, n, sites):
+def test_synthetic_trace_parity(fpx, name, recipe, mode, n, sites, variant):
     p = fpxgen.Params(seed=0x5EED0000 + recipe, n_records=n, n_sites=sites, recipe=recipe, p_fp64=0.5)
     hdr, arena = fpxgen.generate_host(p)
     inj, w = fpxgen.plan_injections(p, 400, flow=(recipe == fpxgen.RECIPE_FLOW))
     fpxgen.apply_host(w, hdr, arena)
     base = 10**12 + 7
-    got, st, stats = gpu_scan(fpx, hdr, arena, base=base, mode=mode)
+    got, st, stats = gpu_scan(fpx, hdr, arena, base=base, mode=mode, flags=variant)
     ref = oracle_scan(hdr, arena, base, mode)
     assert st == fpx.OK and stats.bad_records == 0
     assert_same(got, ref.entries())
@@ -131,25 +133,27 @@ def test_synthetic_trace_parity(fpx, name, recipe, mode, n, sites):
     assert table_dict(got) == expected_from_injections(hdr, inj, base, mode)
 
 
-def test_dense_nan_storm(fpx):
+@pytest.mark.parametrize("variant", [0, 1], ids=["tma", "ldg"])
+def test_dense_nan_storm(fpx, variant):
     p = fpxgen.Params(seed=77, n_records=60_000, n_sites=200, recipe=fpxgen.RECIPE_STRESS, dense_nan=1.0)
     hdr, arena = fpxgen.generate_host(p)
-    got, st, _ = gpu_scan(fpx, hdr, arena)
+    got, st, _ = gpu_scan(fpx, hdr, arena, flags=variant)
     assert_same(got, oracle_scan(hdr, arena).entries())
     p.dense_nan = 0.01
     hdr, arena = fpxgen.generate_host(p)
-    got, st, _ = gpu_scan(fpx, hdr, arena, base=3)
+    got, st, _ = gpu_scan(fpx, hdr, arena, base=3, flags=variant)
     assert_same(got, oracle_scan(hdr, arena, 3).entries())
 
 
+@pytest.mark.parametrize("variant", [0, 1], ids=["tma", "ldg"])
 @pytest.mark.parametrize("n", [1, 31, 32, 33, 255, 257, 4097])
-def test_ragged_sizes(fpx, n):
+def test_ragged_sizes(fpx, n, variant):
     p = fpxgen.Params(seed=n, n_records=n, n_sites=7, recipe=fpxgen.RECIPE_MIX, p_partial=0.5)
     hdr, arena = fpxgen.generate_host(p)
     _, w = fpxgen.plan_injections(p, max(1, n // 8))
     fpxgen.apply_host(w, hdr, arena)
     for mode in (DEST,):
-        got, st, _ = gpu_scan(fpx, hdr, arena, base=n, mode=mode)
+        got, st, _ = gpu_scan(fpx, hdr, arena, base=n, mode=mode, flags=variant)
         assert_same(got, oracle_scan(hdr, arena, n, mode).entries())
 
 

@@ -21,3 +21,12 @@ if [ "${NCU:-1}" = 1 ]; then
      python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline ${NCU_FULL_ARGS:-} > $OUT/ncu_full.log 2>&1; echo "ncu full rc=$?"
   tail -3 $OUT/ncu_full.log
 fi
+if [ -n "${EXTRA:-}" ]; then
+  i=0
+  IFS=';' read -ra CMDS <<< "$EXTRA"
+  for c in "${CMDS[@]}"; do
+    i=$((i+1)); echo "== extra $i: $c" >> $OUT/extra.log
+    timeout 600 bash -c "$c" >> $OUT/extra.log 2>&1; echo "rc=$?" >> $OUT/extra.log
+  done
+  grep -E '^==|^\{|rc=' $OUT/extra.log | cut -c1-400
+fi
