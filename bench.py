@@ -42,6 +42,9 @@ CONFIGS = {
                recipe=2, n=7_800_000, sites=1_000, p_fp64=0.3, mode=1, rho=1e-6),
     "c4a": dict(name="C4a: HADD2/HFMA2/HMUL2 FP16x2/BF16x2 + HMMA records, 1e8 records, 1e3 sites, density 1e-6",
                 recipe=3, n=100_000_000, sites=1_000, p_fp64=0.0, mode=0, rho=1e-6),
+    "c4b": dict(name="C4b: fpx_scan_tensor over 40 GB of BF16 model activations (2e10 torch.randn values), "
+                     "sparse NaN/INF at 1e-7 plus whole-row NaN bursts",
+                kind="tensor", n=20_000_000_000, dtype="bf16", rho=1e-7, sites=1, mode=0, recipe=-1, p_fp64=0.0),
     "c5": dict(name="C5 shard: FP32 dest-only trace, 10^11 lane-values / 8 GPUs = 3.9e8 records per GPU, 1e6 sites",
                recipe=1, n=390_625_000, sites=1_000_000, p_fp64=0.0, mode=0, rho=1e-6),
 }
@@ -177,6 +180,8 @@ def run_reference(args, cfg, seed):
     import fpxgen
     import oracle
 
+    if cfg.get("kind") == "tensor":
+        return run_reference_tensor(args, cfg, seed)
     # each step: a bounded sample of the workload sized to ~0.25 s of oracle time
     probe_n = 20_000
     p = fpxgen.Params(seed=seed, n_records=probe_n, n_sites=cfg["sites"], recipe=cfg["recipe"], p_fp64=cfg["p_fp64"])
@@ -212,6 +217,153 @@ def run_reference(args, cfg, seed):
     }
     print(json.dumps(line), flush=True)
     return 0
+
+
+def run_reference_tensor(args, cfg, seed):
+    """--impl reference for C4b: the oracle's tensor scan on a host sample."""
+    import torch
+
+    import oracle
+
+    g = torch.Generator().manual_seed(seed)
+    n = 1 << 24
+    x = torch.randn(n, generator=g, dtype=torch.float32).to(torch.bfloat16)
+    x[torch.randint(0, n, (max(1, int(cfg["rho"] * n)),), generator=g)] = float("nan")
+    host = x.view(torch.int16).numpy()
+    fmt = {"bf16": 3, "fp16": 2, "fp32": 0}[cfg["dtype"]]
+    for _ in range(args.warmup):
+        oracle.Table().scan_tensor(host, fmt, site=0)
+    dt_total = 0.0
+    for _ in range(args.steps):
+        t = oracle.Table()
+        t0 = time.perf_counter()
+        t.scan_tensor(host, fmt, site=0)
+        dt_total += time.perf_counter() - t0
+    value = n * args.steps / dt_total
+    sample = f"{n} BF16 torch.randn values per step (same recipe as C4b), single-threaded oracle"
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt_total / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u16", "data": "synthetic",
+        "config": {"workload": cfg["name"], "elements_per_step": n},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+    return 0
+
+
+class RecordsWorkload:
+    """A record trace (configs C1-C3, C4a, C5) generated in HBM by fpxgen."""
+
+    def __init__(self, cfg, rank, seed, variant):
+        self.cfg, self.seed = cfg, seed
+        self.p, self.hdr, self.arena, self.planes, self.r0, self.inj = build_trace(cfg, rank, 1, seed)
+        self.lane_values, self.nbytes = workload_stats(self.hdr, cfg["mode"])
+        self.kernel = "k_scan_records_" + variant
+        self._host = None
+
+    def scan(self, h, stream):
+        h.scan_records(self.hdr, self.arena, base_index=self.r0, mode=self.cfg["mode"], stream=stream,
+                       n_records=self.cfg["n"], arena_planes=self.planes)
+
+    def make_host_copies(self):
+        import torch
+
+        hh = torch.empty(self.hdr.shape, dtype=self.hdr.dtype, pin_memory=True)
+        ah = torch.empty(self.arena.shape, dtype=self.arena.dtype, pin_memory=True)
+        hh.copy_(self.hdr)
+        ah.copy_(self.arena)
+        self._host = (hh, ah)
+
+    def h2d(self):
+        hh, ah = self._host
+        self.hdr.copy_(hh, non_blocking=True)
+        self.arena.copy_(ah, non_blocking=True)
+        return hh.numel() * 4 + ah.numel() * 4
+
+    def drop_host_copies(self):
+        self._host = None
+
+    def config(self):
+        return {"records_per_gpu": self.cfg["n"], "sites": self.cfg["sites"],
+                "mode": ["dest", "flow"][self.cfg["mode"]], "planted_events": int(len(self.inj))}
+
+    def cpu_baseline(self):
+        return cpu_baseline_oracle(self.cfg, self.seed)
+
+
+class TensorWorkload:
+    """C4b: a plain activation buffer (torch.randn, seeded) with planted NaN/INF."""
+
+    def __init__(self, cfg, rank, seed, dev):
+        import torch
+
+        self.cfg, self.seed = cfg, seed
+        n = cfg["n"]
+        dt = {"bf16": torch.bfloat16, "fp16": torch.float16, "fp32": torch.float32}[cfg["dtype"]]
+        g = torch.Generator(device=dev).manual_seed(seed + rank)
+        self.x = torch.empty(n, dtype=dt, device=dev)
+        chunk = 1 << 30
+        for a in range(0, n, chunk):  # randn in chunks keeps the fp32 temporaries small
+            b = min(n, a + chunk)
+            self.x[a:b] = torch.randn(b - a, generator=g, device=dev, dtype=torch.float32).to(dt)
+        n_inj = int(round(cfg["rho"] * n))
+        idx = torch.randint(0, n, (n_inj,), generator=g, device=dev)
+        self.x[idx[: n_inj // 2]] = float("nan")
+        self.x[idx[n_inj // 2:]] = float("inf")
+        for r in range(4):  # SRU-style uninitialised rows (P:715): whole 4096-value rows of NaN
+            row = int(torch.randint(0, n // 4096, (1,), generator=g, device=dev)) * 4096
+            self.x[row: row + 4096] = float("nan")
+        self.base = rank * n
+        self.lane_values = n
+        self.nbytes = n * self.x.element_size()
+        self.kernel = "k_scan_tensor"
+        self.planted = n_inj + 4 * 4096
+        self._host = None
+
+    def scan(self, h, stream):
+        h.scan_tensor(self.x, site=0, base_index=self.base, stream=stream)
+
+    def make_host_copies(self):
+        import torch
+
+        self._host = torch.empty(self.x.shape, dtype=self.x.dtype, pin_memory=True)
+        self._host.copy_(self.x)
+
+    def h2d(self):
+        self.x.copy_(self._host, non_blocking=True)
+        return self._host.numel() * self._host.element_size()
+
+    def drop_host_copies(self):
+        self._host = None
+
+    def config(self):
+        return {"elements_per_gpu": self.cfg["n"], "dtype": self.cfg["dtype"], "planted_events": self.planted}
+
+    def cpu_baseline(self, budget_s: float = 12.0):
+        import oracle
+
+        fmt = {"bf16": 3, "fp16": 2, "fp32": 0}[self.cfg["dtype"]]
+        m = 1 << 24
+        host = self.x[:m].view(torch_int_view(self.x)).cpu().numpy()
+        t = oracle.Table()
+        t0 = time.perf_counter()
+        t.scan_tensor(host, fmt, site=0)
+        dt = time.perf_counter() - t0
+        m2 = int(min(self.cfg["n"], m * budget_s / max(dt, 1e-6)))
+        host = self.x[:m2].view(torch_int_view(self.x)).cpu().numpy()
+        t = oracle.Table()
+        t0 = time.perf_counter()
+        t.scan_tensor(host, fmt, site=0)
+        dt = time.perf_counter() - t0
+        return {"value": m2 / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+                "sample": f"first {m2} elements of the same C4b buffer, single-threaded C++ oracle, {dt:.1f} s"}
+
+
+def torch_int_view(x):
+    import torch
+
+    return {2: torch.int16, 4: torch.int32, 8: torch.int64}[x.element_size()]
 
 
 def main():
@@ -251,19 +403,19 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
 
-    p, hdr, arena, planes, r0, inj = build_trace(cfg, rank, world, seed)
-    lane_values, nbytes = workload_stats(hdr, cfg["mode"])
-    torch.cuda.synchronize()
-
     h = fpx.Handle(local, flags=fpx.OPT_SCAN_LDG if args.variant == "ldg" else 0)
     stream = torch.cuda.current_stream(dev)
-    n = cfg["n"]
+    if cfg.get("kind") == "tensor":
+        wl = TensorWorkload(cfg, rank, seed, dev)
+    else:
+        wl = RecordsWorkload(cfg, rank, seed, args.variant)
+    torch.cuda.synchronize()
 
     def step(ev_a=None, ev_b=None):
         h.reset(stream=stream)
         if ev_a is not None:
             ev_a.record(stream)
-        h.scan_records(hdr, arena, base_index=r0, mode=cfg["mode"], stream=stream, n_records=n, arena_planes=planes)
+        wl.scan(h, stream)
         if ev_b is not None:
             ev_b.record(stream)
         if world > 1:
@@ -297,7 +449,6 @@ def main():
         total_ms, kern_ms = float(t[0]), float(t[1])
     ms_per_step = total_ms / K
 
-    # correctness of what was timed: the table equals the planted closed form
     ents = h.fetch()
     ok_status = h.last_status
 
@@ -306,10 +457,7 @@ def main():
     e2e = None
     if not args.no_e2e and world == 1:
         try:
-            hdr_h = torch.empty(hdr.shape, dtype=hdr.dtype, pin_memory=True)
-            arena_h = torch.empty(arena.shape, dtype=arena.dtype, pin_memory=True)
-            hdr_h.copy_(hdr)
-            arena_h.copy_(arena)
+            wl.make_host_copies()
             torch.cuda.synchronize()
             d2h = 0
             e_a, e_b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -317,23 +465,21 @@ def main():
             for i in range(args.e2e_steps + 1):
                 torch.cuda.synchronize()
                 e_a.record(stream)
-                hdr.copy_(hdr_h, non_blocking=True)
-                arena.copy_(arena_h, non_blocking=True)
+                h2d = wl.h2d()
                 h.reset(stream=stream)
-                h.scan_records(hdr, arena, base_index=r0, mode=cfg["mode"], stream=stream, n_records=n,
-                               arena_planes=planes)
+                wl.scan(h, stream)
                 got = h.fetch()  # synchronises; D2H of the entries
                 e_b.record(stream)
                 torch.cuda.synchronize()
                 if i > 0:  # first pass = warm-up
                     tot += e_a.elapsed_time(e_b)
                 d2h = got.nbytes
-            e2e = {"value": lane_values / (tot / args.e2e_steps / 1e3), "unit": UNIT,
-                   "h2d_bytes_per_step": hdr.numel() * 4 + arena.numel() * 4, "d2h_bytes_per_step": int(d2h),
-                   "steps": args.e2e_steps}
-            del hdr_h, arena_h
+            e2e = {"value": wl.lane_values / (tot / args.e2e_steps / 1e3), "unit": UNIT,
+                   "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "steps": args.e2e_steps}
+            wl.drop_host_copies()
         except Exception as ex:  # pragma: no cover - reported, not hidden
             e2e = {"value": None, "unit": UNIT, "error": str(ex)[:200]}
+    lane_values, nbytes = wl.lane_values, wl.nbytes
 
     if rank != 0:
         if world > 1:
@@ -349,7 +495,7 @@ def main():
             tj = json.load(f)
         traffic = tj.get(args.config, {}).get("dram_bytes_per_launch")
     clocks = clk.summary()
-    cpu = None if args.no_cpu_baseline else cpu_baseline_oracle(cfg, seed)
+    cpu = None if args.no_cpu_baseline else wl.cpu_baseline()
     line = {
         "metric": METRIC,
         "value": world * lane_values / (ms_per_step / 1e3),
@@ -365,16 +511,13 @@ def main():
         "data": "synthetic (fpxgen counter-based trace generated in HBM, planted exceptions)",
         "config": {
             "workload": cfg["name"],
-            "records_per_gpu": n,
-            "sites": cfg["sites"],
-            "mode": ["dest", "flow"][cfg["mode"]],
+            **wl.config(),
             "lane_values_per_gpu_step": lane_values,
             "algorithmic_bytes_per_gpu_step": nbytes,
-            "planted_events": int(len(inj)),
             "table_entries": int(len(ents)),
             "fetch_status": int(ok_status),
             "l2": "inputs >> 126 MB L2 (no flush needed)",
-            "parallelism": f"record shards x{world}" + (" + NCCL merge per step" if world > 1 else ""),
+            "parallelism": f"shards x{world}" + (" + NCCL merge per step" if world > 1 else ""),
         },
         "roofline": {
             "bound": "hbm",
@@ -383,7 +526,7 @@ def main():
             "unit": "GB/s",
             "frac": achieved / peak,
             "traffic": traffic,
-            "kernel": "k_scan_records_" + args.variant,
+            "kernel": wl.kernel,
             "kernel_ms": kern_ms,
             "peak_source": peak_src,
         },

@@ -27,6 +27,8 @@
 // ring buys (profiles/).
 #include <cuda_runtime.h>
 
+#include <cstdlib>
+
 #include "fpx_records.cuh"
 
 namespace fpx {
@@ -79,9 +81,12 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 }
 
 // ---- TMA-ring kernel ------------------------------------------------------------
-constexpr int TMA_WARPS = 8;   // warps per CTA (one CTA per SM)
-constexpr int STAGES = 3;      // ring depth per warp (STAGES-1 tiles in flight)
-constexpr int PLANES = 64;     // planes per stage (8 KB)
+// Ring geometry: WARPS warps per CTA (one CTA per SM), STAGES stages per warp
+// (STAGES-1 tiles in flight while one is consumed), PLANES planes per stage.
+template <int WARPS_, int STAGES_, int PLANES_>
+struct RingCfg {
+  static constexpr int WARPS = WARPS_, STAGES = STAGES_, PLANES = PLANES_;
+};
 
 struct StageMeta {
   uint32_t k;                    // records in the tile (0 = no tile)
@@ -90,34 +95,51 @@ struct StageMeta {
   uint64_t gidx0;                // global index of the tile's first record
 };
 
+template <class C>
 struct WarpSmem {
-  uint32_t planes[STAGES][PLANES * 32];  // 128 B per plane
-  uint2 items[STAGES][PLANES];           // {slot, active mask}
-  RecDesc recs[STAGES][TILE];
-  StageMeta meta[STAGES];
-  uint64_t bar[STAGES];
+  uint32_t planes[C::STAGES][C::PLANES * 32];  // 128 B per plane
+  uint2 items[C::STAGES][C::PLANES];           // {slot, active mask}
+  RecDesc recs[C::STAGES][TILE];
+  StageMeta meta[C::STAGES];
+  uint64_t bar[C::STAGES];
 };
-constexpr size_t TMA_SMEM = sizeof(WarpSmem) * TMA_WARPS;
-static_assert(TMA_SMEM <= 227 * 1024, "ring exceeds shared memory");
-
-// Planes of a valid, active record the mode must look at (all contiguous from
-// plane 0 of the record).
-template <int MODE>
-__device__ __forceinline__ uint32_t needed_planes(uint32_t meta) {
-  const uint32_t op = op_of(meta), fmt = fmt_of(meta), dw = dwords_of(meta), ns = nsrc_of(meta);
-  if (op == FPX_OP_DIV) return 0u;  // exact path reads DIV records itself
-  if (MODE == FPX_MODE_DEST) return is_compare(op) ? 0u : dw;
-  return dw + ns * sw_of(fmt);
+template <class C>
+constexpr size_t ring_smem() {
+  return sizeof(WarpSmem<C>) * C::WARPS;
 }
 
+// Fast-path item counts of a valid, active record, packed 4 x 8 bit (byte =
+// format).  The items enumerate exactly the planes the mode must look at
+// (DEST: destination words; FLOW: destination + source words), which are
+// contiguous from plane 0 of the record; an FP64 item is a (lo, hi) pair.
 template <int MODE>
-__global__ void __launch_bounds__(TMA_WARPS * 32, 1)
+__device__ __forceinline__ uint32_t packed_items(uint32_t meta, bool& force) {
+  const uint32_t op = op_of(meta), fmt = fmt_of(meta), dw = dwords_of(meta), ns = nsrc_of(meta);
+  force = op == FPX_OP_DIV;  // DIV0 needs the sources: exact path reads DIV records itself
+  if (force) return 0u;
+  uint32_t n;
+  if (MODE == FPX_MODE_DEST) {
+    if (is_compare(op)) return 0u;
+    n = fmt == FPX_FP64 ? dw / 2 : dw;
+  } else {
+    n = fmt == FPX_FP64 ? (dw + 2 * ns) / 2 : dw + ns;
+  }
+  return n << (8 * fmt);
+}
+// planes covered by packed item counts (an FP64 item spans two planes)
+__device__ __forceinline__ uint32_t planes_of_items(uint32_t p) {
+  return (p & 0xFFu) + 2u * ((p >> 8) & 0xFFu) + ((p >> 16) & 0xFFu) + (p >> 24);
+}
+
+template <int MODE, class C>
+__global__ void __launch_bounds__(C::WARPS * 32, 1)
 k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __restrict__ arena,
                    uint64_t arena_planes, uint64_t base_index, uint64_t recs_per_warp, const TableView tv) {
+  constexpr int STAGES = C::STAGES, PLANES = C::PLANES;
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  WarpSmem& sm = reinterpret_cast<WarpSmem*>(smem_raw)[warp];
-  const uint64_t gw = blockIdx.x * (uint64_t)TMA_WARPS + warp;
+  WarpSmem<C>& sm = reinterpret_cast<WarpSmem<C>*>(smem_raw)[warp];
+  const uint64_t gw = blockIdx.x * (uint64_t)C::WARPS + warp;
   const uint64_t start = gw * recs_per_warp;
   if (start >= n) return;  // warp-uniform; no block-wide barriers below
   const uint64_t end = min(n, start + recs_per_warp);
@@ -147,40 +169,34 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const bool inrange = cursor + lane < end;
     const bool ok = inrange && record_valid<MODE>(h, arena_planes);
     const uint32_t mask = ok ? h.y : 0u;
-    const uint32_t c = (ok && mask != 0u) ? needed_planes<MODE>(h.z) : 0u;
-    uint32_t incl = c;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t t = __shfl_up_sync(FULL, incl, o);
-      if (lane >= o) incl += t;
-    }
-    // the tile = leading records whose planes fit the stage (>= 1 record)
-    const uint32_t k = __popc(__ballot_sync(FULL, inrange && incl <= (uint32_t)PLANES));
-    const bool in_tile = (uint32_t)lane < k;
-    const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
-    if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
-    const uint32_t cc = in_tile ? c : 0u;
-    const uint32_t slot = incl - c;
-    const uint32_t total = __shfl_sync(FULL, incl, k - 1);
     bool force = false;
-    const uint32_t cnt = item_counts<MODE>(h.z, in_tile && ok && mask != 0u, force);
-
-    // items: exclusive scan of the packed per-format counts
+    const uint32_t cnt = (ok && mask != 0u) ? packed_items<MODE>(h.z, force) : 0u;
+    // one warp scan of the packed counts gives item positions and plane slots
     uint32_t ic = cnt;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
       const uint32_t t = __shfl_up_sync(FULL, ic, o);
       if (lane >= o) ic += t;
     }
-    const uint32_t itot = __shfl_sync(FULL, ic, 31);
+    const uint32_t incl_planes = planes_of_items(ic);
+    // the tile = leading records whose planes fit the stage (>= 1 record)
+    const uint32_t k = __popc(__ballot_sync(FULL, inrange && incl_planes <= (uint32_t)PLANES));
+    const bool in_tile = (uint32_t)lane < k;
+    const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
+    if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
+    const uint32_t c = in_tile ? planes_of_items(cnt) : 0u;
+    const uint32_t slot = incl_planes - planes_of_items(cnt);
+    const uint32_t itot = __shfl_sync(FULL, ic, k - 1);
+    const uint32_t total = planes_of_items(itot);
     const uint32_t iex = ic - cnt;
     const uint32_t n32 = itot & 0xFFu, n64 = (itot >> 8) & 0xFFu, n16 = (itot >> 16) & 0xFFu, nb16 = itot >> 24;
+    const bool force_any = __any_sync(FULL, in_tile && force);
     // the ring slot may still be read by the previous consume of this stage:
     // order those generic reads before the async-proxy writes below
     __syncwarp();
     fence_proxy_async_smem();
     sm.recs[s][lane] = in_tile ? RecDesc{h.w, mask, h.z, h.x} : RecDesc{0u, 0u, 0u, 0u};
-    if (cnt != 0u) {
+    if (in_tile && cnt != 0u) {
       const uint32_t fmt = fmt_of(h.z);
       const uint32_t my = (cnt >> (8 * fmt)) & 0xFFu;
       const uint32_t seg = fmt == 0u ? 0u : fmt == 1u ? n32 : fmt == 2u ? n32 + n64 : n32 + n64 + n16;
@@ -188,7 +204,6 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       const uint32_t step = fmt == FPX_FP64 ? 2u : 1u;
       for (uint32_t q = 0; q < my; ++q) sm.items[s][at + q] = make_uint2(slot + q * step, mask);
     }
-    const bool force_any = __any_sync(FULL, force);
     if (lane == 0) {
       m.k = k;
       m.n32 = n32;
@@ -200,9 +215,9 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     }
     // runs of arena-adjacent records -> one bulk copy each
     const uint32_t a = h.w;
-    const uint32_t prev_end = __shfl_up_sync(FULL, a + cc, 1);
-    const uint32_t prev_c = __shfl_up_sync(FULL, cc, 1);
-    const bool head = cc != 0u && (lane == 0 || prev_c == 0u || prev_end != a);
+    const uint32_t prev_end = __shfl_up_sync(FULL, a + c, 1);
+    const uint32_t prev_c = __shfl_up_sync(FULL, c, 1);
+    const bool head = c != 0u && (lane == 0 || prev_c == 0u || prev_end != a);
     const uint32_t heads = __ballot_sync(FULL, head);
     const uint32_t above = lane == 31 ? 0u : heads & (0xFFFFFFFFu << (lane + 1));  // heads above this lane
     const uint32_t next = above ? (uint32_t)(__ffs(above) - 1) : 32u;
@@ -231,14 +246,14 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     phase ^= 1u << s;
 
     // ---- fast path over the staged planes --------------------------------
-    const uint32_t* __restrict__ pl = sm.planes[s];
+    const uint32_t* __restrict__ pl = sm.planes[s] + lane;
     const uint2* __restrict__ it = sm.items[s];
     uint32_t mn32 = 0xFFFFFFFFu, mx32 = 0u, mn64 = 0xFFFFFFFFu, mx64 = 0u;
     uint32_t mn16 = 0xFFFFFFFFu, mx16 = 0u, mnb = 0xFFFFFFFFu, mxb = 0u;
 #pragma unroll 4
     for (uint32_t q = 0; q < m.n32; ++q) {
       const uint2 t = it[q];
-      const uint32_t x = pl[t.x * 32 + lane] & 0x7FFFFFFFu & lane_ext(t.y, lane);
+      const uint32_t x = pl[t.x * 32] & 0x7FFFFFFFu & lane_ext(t.y, lane);
       mn32 = min(mn32, x - 1u);  // < 0x7FFFFF  <=> subnormal
       mx32 = max(mx32, x);       // > 0x7F7FFFFF <=> INF / NaN
     }
@@ -246,8 +261,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     for (uint32_t q = 0; q < m.n64; ++q) {
       const uint2 t = it[m.n32 + q];
       const uint32_t e = lane_ext(t.y, lane);
-      const uint32_t lo = pl[t.x * 32 + lane] & e;
-      const uint32_t ah = pl[(t.x + 1) * 32 + lane] & 0x7FFFFFFFu & e;
+      const uint32_t lo = pl[t.x * 32] & e;
+      const uint32_t ah = pl[t.x * 32 + 32] & 0x7FFFFFFFu & e;
       const uint32_t a2 = (ah << 1) | min(lo, 1u);  // 0 zero, [1,0x1FFFFF] SUB, >= 0xFFE00000 INF/NaN
       mn64 = min(mn64, a2 - 1u);
       mx64 = max(mx64, a2);
@@ -255,7 +270,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 #pragma unroll 4
     for (uint32_t q = 0; q < m.n16 + m.nb16; ++q) {
       const uint2 t = it[m.n32 + m.n64 + q];
-      const uint32_t x = pl[t.x * 32 + lane] & 0x7FFF7FFFu & lane_ext(t.y, lane);
+      const uint32_t x = pl[t.x * 32] & 0x7FFF7FFFu & lane_ext(t.y, lane);
       const uint32_t l = x & 0xFFFFu, hh = x >> 16;
       if (q < m.n16) {
         mn16 = min(mn16, min(l - 1u, hh - 1u));
@@ -269,6 +284,39 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
                      mn16 < 0x03FFu || mx16 > 0x7BFFu || mnb < 0x007Fu || mxb > 0x7F7Fu;
     if (__any_sync(FULL, hit) || m.force) exact_tile<MODE>(sm.recs[s], lane_base, lane, m.gidx0, tv);
   }
+}
+
+// Ring configurations compiled in; FPX_RING (environment, tuning only) picks
+// one, default RING_DEFAULT.
+using Ring0 = RingCfg<16, 2, 48>;
+using Ring1 = RingCfg<8, 3, 64>;
+using Ring2 = RingCfg<12, 2, 64>;
+using Ring3 = RingCfg<16, 2, 32>;
+static_assert(ring_smem<Ring0>() <= 227 * 1024 && ring_smem<Ring1>() <= 227 * 1024 &&
+                  ring_smem<Ring2>() <= 227 * 1024 && ring_smem<Ring3>() <= 227 * 1024,
+              "ring exceeds shared memory");
+
+template <int MODE, class C>
+cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uint64_t arena_planes, uint64_t base_index,
+                        const TableView& tv, int num_sms, cudaStream_t s) {
+  static bool attr_set[64] = {};  // per device
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 64 || !attr_set[dev]) {
+    cudaError_t e = cudaFuncSetAttribute(k_scan_records_tma<MODE, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)ring_smem<C>());
+    if (e != cudaSuccess) return e;
+    if (dev < 64) attr_set[dev] = true;
+  }
+  // one CTA per SM; each warp a contiguous range of records (whole tiles of 32
+  // where possible, so that ranges stay 512-B aligned in the header array)
+  const uint64_t warps = (uint64_t)num_sms * C::WARPS;
+  uint64_t per = (n + warps - 1) / warps;
+  per = (per + TILE - 1) / TILE * TILE;
+  const uint64_t blocks = ((n + per - 1) / per + C::WARPS - 1) / C::WARPS;
+  k_scan_records_tma<MODE, C><<<(unsigned)blocks, C::WARPS * 32, ring_smem<C>(), s>>>(hdr, n, arena, arena_planes,
+                                                                                      base_index, per, tv);
+  return cudaGetLastError();
 }
 
 // ---- register-staged LDG kernel (ablation) ------------------------------------
@@ -423,24 +471,18 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
                                                                          d_arena, arena_planes, base_index, tv);
     return cudaGetLastError();
   }
-  static bool attr_set[64] = {};  // per device
-  int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev >= 64 || !attr_set[dev]) {
-    cudaError_t e = cudaFuncSetAttribute(k_scan_records_tma<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)TMA_SMEM);
-    if (e != cudaSuccess) return e;
-    if (dev < 64) attr_set[dev] = true;
+  static int ring = -1;
+  if (ring < 0) {
+    const char* e = getenv("FPX_RING");
+    ring = e ? atoi(e) : 0;
   }
-  // one CTA per SM; each warp a contiguous range of records (whole tiles of 32
-  // where possible, so that ranges stay 512-B aligned in the header array)
-  const uint64_t warps = (uint64_t)num_sms * TMA_WARPS;
-  uint64_t per = (n + warps - 1) / warps;
-  per = (per + TILE - 1) / TILE * TILE;
-  const uint64_t blocks = ((n + per - 1) / per + TMA_WARPS - 1) / TMA_WARPS;
-  k_scan_records_tma<MODE><<<(unsigned)blocks, TMA_WARPS * 32, TMA_SMEM, s>>>(
-      reinterpret_cast<const uint4*>(d_hdr), n, d_arena, arena_planes, base_index, per, tv);
-  return cudaGetLastError();
+  const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
+  switch (ring) {
+    case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
+    case 2: return launch_ring<MODE, Ring2>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
+    case 3: return launch_ring<MODE, Ring3>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
+    default: return launch_ring<MODE, Ring0>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
+  }
 }
 
 }  // namespace

@@ -30,3 +30,7 @@ if [ -n "${EXTRA:-}" ]; then
   done
   grep -E '^==|^\{|rc=' $OUT/extra.log | cut -c1-400
 fi
+if [ "${NCU_TENSOR:-0}" = 1 ]; then
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_scan_tensor -s 3 -c 1 -o $OUT/prof_tensor \
+     python bench.py --config c4b --records 1000000000 --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > $OUT/ncu_tensor.log 2>&1; echo "ncu tensor rc=$?"
+fi
