@@ -92,14 +92,17 @@ struct StageMeta {
   uint32_t k;                    // records in the tile (0 = no tile)
   uint32_t n32, n64, n16, nb16;  // fast-path items per list
   uint32_t force;                // tile holds a record that must take the exact path
+  uint32_t partial;              // bit j: record j has a partial active mask
+  uint32_t pad;
   uint64_t gidx0;                // global index of the tile's first record
 };
 
 template <class C>
 struct WarpSmem {
   uint32_t planes[C::STAGES][C::PLANES * 32];  // 128 B per plane
-  uint2 items[C::STAGES][C::PLANES];           // {slot, active mask}
+  uint32_t items[C::STAGES][C::PLANES];        // plane slot of each fast-path item
   RecDesc recs[C::STAGES][TILE];
+  uint32_t span[C::STAGES][TILE];              // slot | planes << 16 of each record
   StageMeta meta[C::STAGES];
   uint64_t bar[C::STAGES];
 };
@@ -202,9 +205,12 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       const uint32_t seg = fmt == 0u ? 0u : fmt == 1u ? n32 : fmt == 2u ? n32 + n64 : n32 + n64 + n16;
       const uint32_t at = seg + ((iex >> (8 * fmt)) & 0xFFu);
       const uint32_t step = fmt == FPX_FP64 ? 2u : 1u;
-      for (uint32_t q = 0; q < my; ++q) sm.items[s][at + q] = make_uint2(slot + q * step, mask);
+      for (uint32_t q = 0; q < my; ++q) sm.items[s][at + q] = slot + q * step;
     }
+    sm.span[s][lane] = slot | (c << 16);
+    const uint32_t partial = __ballot_sync(FULL, c != 0u && mask != FULL);
     if (lane == 0) {
+      m.partial = partial;
       m.k = k;
       m.n32 = n32;
       m.n64 = n64;
@@ -245,32 +251,42 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     mbar_wait(&sm.bar[s], (phase >> s) & 1u);
     phase ^= 1u << s;
 
+    // inactive lanes of partial-mask records: zero their words once (zero is
+    // clean in every format), so the fast path below needs no per-item mask
+    uint32_t* __restrict__ pl = sm.planes[s] + lane;
+    for (uint32_t pm = m.partial; pm != 0u; pm &= pm - 1u) {
+      const int j = __ffs(pm) - 1;
+      if (((sm.recs[s][j].mask >> lane) & 1u) == 0u) {
+        const uint32_t sp = sm.span[s][j];
+        for (uint32_t q = 0; q < (sp >> 16); ++q) pl[((sp & 0xFFFFu) + q) * 32] = 0u;
+      }
+    }
+    __syncwarp();
+
     // ---- fast path over the staged planes --------------------------------
-    const uint32_t* __restrict__ pl = sm.planes[s] + lane;
-    const uint2* __restrict__ it = sm.items[s];
+    // witnesses (no false negatives, exact):
+    //   FP32  a2 = |x| << 1:  subnormal <=> a2 - 2 < 0xFFFFFE;  INF/NaN <=> a2 >= 0xFF000000
+    //   FP64  a3 = |hi| | (lo != 0):  subnormal <=> a3 - 1 < 0xFFFFF;  INF/NaN <=> a3 >= 0x7FF00000
+    //   FP16 / BF16 per half:  subnormal <=> h - 1 < 0x3FF / 0x7F;  INF/NaN <=> h >= 0x7C00 / 0x7F80
+    const uint32_t* __restrict__ it = sm.items[s];
     uint32_t mn32 = 0xFFFFFFFFu, mx32 = 0u, mn64 = 0xFFFFFFFFu, mx64 = 0u;
     uint32_t mn16 = 0xFFFFFFFFu, mx16 = 0u, mnb = 0xFFFFFFFFu, mxb = 0u;
 #pragma unroll 4
     for (uint32_t q = 0; q < m.n32; ++q) {
-      const uint2 t = it[q];
-      const uint32_t x = pl[t.x * 32] & 0x7FFFFFFFu & lane_ext(t.y, lane);
-      mn32 = min(mn32, x - 1u);  // < 0x7FFFFF  <=> subnormal
-      mx32 = max(mx32, x);       // > 0x7F7FFFFF <=> INF / NaN
+      const uint32_t a2 = pl[it[q] * 32] << 1;
+      mn32 = min(mn32, a2 - 2u);
+      mx32 = max(mx32, a2);
     }
 #pragma unroll 4
     for (uint32_t q = 0; q < m.n64; ++q) {
-      const uint2 t = it[m.n32 + q];
-      const uint32_t e = lane_ext(t.y, lane);
-      const uint32_t lo = pl[t.x * 32] & e;
-      const uint32_t ah = pl[t.x * 32 + 32] & 0x7FFFFFFFu & e;
-      const uint32_t a2 = (ah << 1) | min(lo, 1u);  // 0 zero, [1,0x1FFFFF] SUB, >= 0xFFE00000 INF/NaN
-      mn64 = min(mn64, a2 - 1u);
-      mx64 = max(mx64, a2);
+      const uint32_t t = it[m.n32 + q] * 32;
+      const uint32_t a3 = (pl[t + 32] & 0x7FFFFFFFu) | min(pl[t], 1u);
+      mn64 = min(mn64, a3 - 1u);
+      mx64 = max(mx64, a3);
     }
 #pragma unroll 4
     for (uint32_t q = 0; q < m.n16 + m.nb16; ++q) {
-      const uint2 t = it[m.n32 + m.n64 + q];
-      const uint32_t x = pl[t.x * 32] & 0x7FFF7FFFu & lane_ext(t.y, lane);
+      const uint32_t x = pl[it[m.n32 + m.n64 + q] * 32] & 0x7FFF7FFFu;
       const uint32_t l = x & 0xFFFFu, hh = x >> 16;
       if (q < m.n16) {
         mn16 = min(mn16, min(l - 1u, hh - 1u));
@@ -280,7 +296,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
         mxb = max(mxb, max(l, hh));
       }
     }
-    const bool hit = mn32 < 0x007FFFFFu || mx32 > 0x7F7FFFFFu || mn64 < 0x001FFFFFu || mx64 >= 0xFFE00000u ||
+    const bool hit = mn32 < 0x00FFFFFEu || mx32 >= 0xFF000000u || mn64 < 0x000FFFFFu || mx64 >= 0x7FF00000u ||
                      mn16 < 0x03FFu || mx16 > 0x7BFFu || mnb < 0x007Fu || mxb > 0x7F7Fu;
     if (__any_sync(FULL, hit) || m.force) exact_tile<MODE>(sm.recs[s], lane_base, lane, m.gidx0, tv);
   }
