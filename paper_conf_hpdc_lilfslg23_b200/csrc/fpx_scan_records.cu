@@ -88,21 +88,23 @@ struct RingCfg {
   static constexpr int WARPS = WARPS_, STAGES = STAGES_, PLANES = PLANES_;
 };
 
+// Fast-path item lists of a stage: 4 formats x {full active mask, partial
+// active mask}.  List index = 2 * fmt + partial.
+constexpr int NLISTS = 8;
+
 struct StageMeta {
-  uint32_t k;                    // records in the tile (0 = no tile)
-  uint32_t n32, n64, n16, nb16;  // fast-path items per list
-  uint32_t force;                // tile holds a record that must take the exact path
-  uint32_t partial;              // bit j: record j has a partial active mask
-  uint32_t pad;
-  uint64_t gidx0;                // global index of the tile's first record
+  uint32_t k;              // records in the tile (0 = no tile)
+  uint32_t force;          // tile holds a record that must take the exact path
+  uint64_t gidx0;          // global index of the tile's first record
+  uint32_t seg[NLISTS + 1];  // list l = items [seg[l], seg[l+1])
+  uint32_t pad[3];
 };
 
 template <class C>
 struct WarpSmem {
   uint32_t planes[C::STAGES][C::PLANES * 32];  // 128 B per plane
-  uint32_t items[C::STAGES][C::PLANES];        // plane slot of each fast-path item
+  uint2 items[C::STAGES][C::PLANES];           // {plane slot, active mask}
   RecDesc recs[C::STAGES][TILE];
-  uint32_t span[C::STAGES][TILE];              // slot | planes << 16 of each record
   StageMeta meta[C::STAGES];
   uint64_t bar[C::STAGES];
 };
@@ -111,28 +113,60 @@ constexpr size_t ring_smem() {
   return sizeof(WarpSmem<C>) * C::WARPS;
 }
 
-// Fast-path item counts of a valid, active record, packed 4 x 8 bit (byte =
-// format).  The items enumerate exactly the planes the mode must look at
-// (DEST: destination words; FLOW: destination + source words), which are
-// contiguous from plane 0 of the record; an FP64 item is a (lo, hi) pair.
+// Fast-path item count of a valid, active record.  The items enumerate
+// exactly the planes the mode must look at (DEST: destination words; FLOW:
+// destination + source words), contiguous from plane 0 of the record; an
+// FP64 item is a (lo, hi) pair of planes.
 template <int MODE>
-__device__ __forceinline__ uint32_t packed_items(uint32_t meta, bool& force) {
+__device__ __forceinline__ uint32_t record_items(uint32_t meta, bool& force) {
   const uint32_t op = op_of(meta), fmt = fmt_of(meta), dw = dwords_of(meta), ns = nsrc_of(meta);
-  force = op == FPX_OP_DIV;  // DIV0 needs the sources: exact path reads DIV records itself
+  force = op == FPX_OP_DIV;  // DIV0 needs the sources: the exact path reads DIV records itself
   if (force) return 0u;
-  uint32_t n;
   if (MODE == FPX_MODE_DEST) {
     if (is_compare(op)) return 0u;
-    n = fmt == FPX_FP64 ? dw / 2 : dw;
-  } else {
-    n = fmt == FPX_FP64 ? (dw + 2 * ns) / 2 : dw + ns;
+    return fmt == FPX_FP64 ? dw / 2 : dw;
   }
-  return n << (8 * fmt);
+  return fmt == FPX_FP64 ? (dw + 2 * ns) / 2 : dw + ns;
 }
-// planes covered by packed item counts (an FP64 item spans two planes)
+// planes covered by packed item counts (bytes: FP32, FP64 pairs, FP16, BF16)
 __device__ __forceinline__ uint32_t planes_of_items(uint32_t p) {
   return (p & 0xFFu) + 2u * ((p >> 8) & 0xFFu) + ((p >> 16) & 0xFFu) + (p >> 24);
 }
+
+// Witness updates (no false negatives, exact thresholds in `hit` below).
+//   FP32  a2 = |x| << 1:  subnormal <=> a2 - 2 < 0xFFFFFE;  INF/NaN <=> a2 >= 0xFF000000
+//   FP64  a3 = |hi| | (lo != 0):  subnormal <=> a3 - 1 < 0xFFFFF;  INF/NaN <=> a3 >= 0x7FF00000
+//   FP16 / BF16 per half:  subnormal <=> h - 1 < 0x3FF / 0x7F;  INF/NaN <=> h >= 0x7C00 / 0x7F80
+// `e` masks inactive lanes to zero (zero is clean in every format).
+struct Witness {
+  uint32_t mn32 = 0xFFFFFFFFu, mx32 = 0u, mn64 = 0xFFFFFFFFu, mx64 = 0u;
+  uint32_t mn16 = 0xFFFFFFFFu, mx16 = 0u, mnb = 0xFFFFFFFFu, mxb = 0u;
+  __device__ __forceinline__ void fp32(uint32_t x) {
+    const uint32_t a2 = x << 1;
+    mn32 = min(mn32, a2 - 2u);
+    mx32 = max(mx32, a2);
+  }
+  __device__ __forceinline__ void fp64(uint32_t lo, uint32_t hi) {
+    const uint32_t a3 = (hi & 0x7FFFFFFFu) | min(lo, 1u);
+    mn64 = min(mn64, a3 - 1u);
+    mx64 = max(mx64, a3);
+  }
+  __device__ __forceinline__ void half2(uint32_t x, bool bf) {
+    x &= 0x7FFF7FFFu;
+    const uint32_t l = x & 0xFFFFu, h = x >> 16;
+    if (bf) {
+      mnb = min(mnb, min(l - 1u, h - 1u));
+      mxb = max(mxb, max(l, h));
+    } else {
+      mn16 = min(mn16, min(l - 1u, h - 1u));
+      mx16 = max(mx16, max(l, h));
+    }
+  }
+  __device__ __forceinline__ bool hit() const {
+    return mn32 < 0x00FFFFFEu || mx32 >= 0xFF000000u || mn64 < 0x000FFFFFu || mx64 >= 0x7FF00000u ||
+           mn16 < 0x03FFu || mx16 > 0x7BFFu || mnb < 0x007Fu || mxb > 0x7F7Fu;
+  }
+};
 
 template <int MODE, class C>
 __global__ void __launch_bounds__(C::WARPS * 32, 1)
@@ -173,51 +207,57 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const bool ok = inrange && record_valid<MODE>(h, arena_planes);
     const uint32_t mask = ok ? h.y : 0u;
     bool force = false;
-    const uint32_t cnt = (ok && mask != 0u) ? packed_items<MODE>(h.z, force) : 0u;
-    // one warp scan of the packed counts gives item positions and plane slots
-    uint32_t ic = cnt;
+    const uint32_t fmt = fmt_of(h.z);
+    const uint32_t ni = (ok && mask != 0u) ? record_items<MODE>(h.z, force) : 0u;
+    const bool part = mask != FULL;
+    // two packed scans (full-mask / partial-mask records; byte = format)
+    const uint32_t cf = part ? 0u : ni << (8 * fmt), cp = part ? ni << (8 * fmt) : 0u;
+    uint32_t sf = cf, sp = cp;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t t = __shfl_up_sync(FULL, ic, o);
-      if (lane >= o) ic += t;
+      const uint32_t tf = __shfl_up_sync(FULL, sf, o), tp = __shfl_up_sync(FULL, sp, o);
+      if (lane >= o) { sf += tf; sp += tp; }
     }
-    const uint32_t incl_planes = planes_of_items(ic);
+    const uint32_t incl_planes = planes_of_items(sf) + planes_of_items(sp);
     // the tile = leading records whose planes fit the stage (>= 1 record)
     const uint32_t k = __popc(__ballot_sync(FULL, inrange && incl_planes <= (uint32_t)PLANES));
     const bool in_tile = (uint32_t)lane < k;
     const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
     if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
-    const uint32_t c = in_tile ? planes_of_items(cnt) : 0u;
-    const uint32_t slot = incl_planes - planes_of_items(cnt);
-    const uint32_t itot = __shfl_sync(FULL, ic, k - 1);
-    const uint32_t total = planes_of_items(itot);
-    const uint32_t iex = ic - cnt;
-    const uint32_t n32 = itot & 0xFFu, n64 = (itot >> 8) & 0xFFu, n16 = (itot >> 16) & 0xFFu, nb16 = itot >> 24;
+    const uint32_t my_planes = planes_of_items(cf + cp);
+    const uint32_t c = in_tile ? my_planes : 0u;
+    const uint32_t slot = incl_planes - my_planes;
+    const uint32_t tf = __shfl_sync(FULL, sf, k - 1), tp = __shfl_sync(FULL, sp, k - 1);
+    const uint32_t total = planes_of_items(tf) + planes_of_items(tp);
     const bool force_any = __any_sync(FULL, in_tile && force);
     // the ring slot may still be read by the previous consume of this stage:
     // order those generic reads before the async-proxy writes below
     __syncwarp();
     fence_proxy_async_smem();
     sm.recs[s][lane] = in_tile ? RecDesc{h.w, mask, h.z, h.x} : RecDesc{0u, 0u, 0u, 0u};
-    if (in_tile && cnt != 0u) {
-      const uint32_t fmt = fmt_of(h.z);
-      const uint32_t my = (cnt >> (8 * fmt)) & 0xFFu;
-      const uint32_t seg = fmt == 0u ? 0u : fmt == 1u ? n32 : fmt == 2u ? n32 + n64 : n32 + n64 + n16;
-      const uint32_t at = seg + ((iex >> (8 * fmt)) & 0xFFu);
+    // list l = 2*fmt + partial starts after all lists of lower formats
+    const uint32_t tot_f = tf + tp;  // per-format item totals (packed)
+    if (in_tile && ni != 0u) {
+      const uint32_t below = (0x00000000u + (fmt > 0 ? (tot_f & 0xFFu) : 0u) + (fmt > 1 ? ((tot_f >> 8) & 0xFFu) : 0u) +
+                              (fmt > 2 ? ((tot_f >> 16) & 0xFFu) : 0u));
+      const uint32_t at = below + (part ? ((tf >> (8 * fmt)) & 0xFFu) : 0u) +
+                          (((part ? sp - cp : sf - cf) >> (8 * fmt)) & 0xFFu);
       const uint32_t step = fmt == FPX_FP64 ? 2u : 1u;
-      for (uint32_t q = 0; q < my; ++q) sm.items[s][at + q] = slot + q * step;
+      for (uint32_t q = 0; q < ni; ++q) sm.items[s][at + q] = make_uint2(slot + q * step, mask);
     }
-    sm.span[s][lane] = slot | (c << 16);
-    const uint32_t partial = __ballot_sync(FULL, c != 0u && mask != FULL);
     if (lane == 0) {
-      m.partial = partial;
       m.k = k;
-      m.n32 = n32;
-      m.n64 = n64;
-      m.n16 = n16;
-      m.nb16 = nb16;
       m.force = force_any ? 1u : 0u;
       m.gidx0 = base_index + cursor;
+      uint32_t acc = 0;
+#pragma unroll
+      for (int f = 0; f < 4; ++f) {
+        m.seg[2 * f] = acc;
+        acc += (tf >> (8 * f)) & 0xFFu;
+        m.seg[2 * f + 1] = acc;
+        acc += (tp >> (8 * f)) & 0xFFu;
+      }
+      m.seg[NLISTS] = acc;
     }
     // runs of arena-adjacent records -> one bulk copy each
     const uint32_t a = h.w;
@@ -246,59 +286,42 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   for (uint32_t i = 0;; ++i) {
     const int s = (int)(i % STAGES);
     produce((int)((i + STAGES - 1) % STAGES));
-    const StageMeta m = sm.meta[s];
-    if (m.k == 0u) break;
+    const StageMeta& m = sm.meta[s];
+    const uint32_t k = m.k;
+    if (k == 0u) break;
     mbar_wait(&sm.bar[s], (phase >> s) & 1u);
     phase ^= 1u << s;
 
-    // inactive lanes of partial-mask records: zero their words once (zero is
-    // clean in every format), so the fast path below needs no per-item mask
-    uint32_t* __restrict__ pl = sm.planes[s] + lane;
-    for (uint32_t pm = m.partial; pm != 0u; pm &= pm - 1u) {
-      const int j = __ffs(pm) - 1;
-      if (((sm.recs[s][j].mask >> lane) & 1u) == 0u) {
-        const uint32_t sp = sm.span[s][j];
-        for (uint32_t q = 0; q < (sp >> 16); ++q) pl[((sp & 0xFFFFu) + q) * 32] = 0u;
-      }
-    }
-    __syncwarp();
-
     // ---- fast path over the staged planes --------------------------------
-    // witnesses (no false negatives, exact):
-    //   FP32  a2 = |x| << 1:  subnormal <=> a2 - 2 < 0xFFFFFE;  INF/NaN <=> a2 >= 0xFF000000
-    //   FP64  a3 = |hi| | (lo != 0):  subnormal <=> a3 - 1 < 0xFFFFF;  INF/NaN <=> a3 >= 0x7FF00000
-    //   FP16 / BF16 per half:  subnormal <=> h - 1 < 0x3FF / 0x7F;  INF/NaN <=> h >= 0x7C00 / 0x7F80
-    const uint32_t* __restrict__ it = sm.items[s];
-    uint32_t mn32 = 0xFFFFFFFFu, mx32 = 0u, mn64 = 0xFFFFFFFFu, mx64 = 0u;
-    uint32_t mn16 = 0xFFFFFFFFu, mx16 = 0u, mnb = 0xFFFFFFFFu, mxb = 0u;
+    const uint32_t* __restrict__ pl = sm.planes[s] + lane;
+    const uint2* __restrict__ it = sm.items[s];
+    uint32_t seg[NLISTS + 1];
+#pragma unroll
+    for (int l = 0; l <= NLISTS; ++l) seg[l] = m.seg[l];
+    Witness w;
 #pragma unroll 4
-    for (uint32_t q = 0; q < m.n32; ++q) {
-      const uint32_t a2 = pl[it[q] * 32] << 1;
-      mn32 = min(mn32, a2 - 2u);
-      mx32 = max(mx32, a2);
+    for (uint32_t q = seg[0]; q < seg[1]; ++q) w.fp32(pl[it[q].x * 32]);
+    for (uint32_t q = seg[1]; q < seg[2]; ++q) {
+      const uint2 t = it[q];
+      w.fp32(pl[t.x * 32] & lane_ext(t.y, lane));
     }
 #pragma unroll 4
-    for (uint32_t q = 0; q < m.n64; ++q) {
-      const uint32_t t = it[m.n32 + q] * 32;
-      const uint32_t a3 = (pl[t + 32] & 0x7FFFFFFFu) | min(pl[t], 1u);
-      mn64 = min(mn64, a3 - 1u);
-      mx64 = max(mx64, a3);
+    for (uint32_t q = seg[2]; q < seg[3]; ++q) {
+      const uint32_t t = it[q].x * 32;
+      w.fp64(pl[t], pl[t + 32]);
     }
-#pragma unroll 4
-    for (uint32_t q = 0; q < m.n16 + m.nb16; ++q) {
-      const uint32_t x = pl[it[m.n32 + m.n64 + q] * 32] & 0x7FFF7FFFu;
-      const uint32_t l = x & 0xFFFFu, hh = x >> 16;
-      if (q < m.n16) {
-        mn16 = min(mn16, min(l - 1u, hh - 1u));
-        mx16 = max(mx16, max(l, hh));
-      } else {
-        mnb = min(mnb, min(l - 1u, hh - 1u));
-        mxb = max(mxb, max(l, hh));
-      }
+    for (uint32_t q = seg[3]; q < seg[4]; ++q) {
+      const uint2 t = it[q];
+      const uint32_t e = lane_ext(t.y, lane);
+      w.fp64(pl[t.x * 32] & e, pl[t.x * 32 + 32] & e);
     }
-    const bool hit = mn32 < 0x00FFFFFEu || mx32 >= 0xFF000000u || mn64 < 0x000FFFFFu || mx64 >= 0x7FF00000u ||
-                     mn16 < 0x03FFu || mx16 > 0x7BFFu || mnb < 0x007Fu || mxb > 0x7F7Fu;
-    if (__any_sync(FULL, hit) || m.force) exact_tile<MODE>(sm.recs[s], lane_base, lane, m.gidx0, tv);
+    for (uint32_t q = seg[4]; q < seg[8]; ++q) {
+      const uint2 t = it[q];
+      const bool partial = (q >= seg[5] && q < seg[6]) || q >= seg[7];
+      const uint32_t e = partial ? lane_ext(t.y, lane) : 0xFFFFFFFFu;
+      w.half2(pl[t.x * 32] & e, q >= seg[6]);
+    }
+    if (__any_sync(FULL, w.hit()) || m.force) exact_tile<MODE>(sm.recs[s], lane_base, lane, m.gidx0, tv);
   }
 }
 
