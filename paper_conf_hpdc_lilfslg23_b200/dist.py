@@ -40,22 +40,26 @@ def merge(keys: torch.Tensor, counts: torch.Tensor, firsts: torch.Tensor, ops, g
     """
     world = dist.get_world_size(group)
     dev = keys.device
-    n = torch.tensor([keys.numel()], dtype=torch.int64, device=dev)
+    # NCCL moves device tensors over NVLink; gloo (CPU tests, or several
+    # ranks sharing one GPU) needs host tensors
+    comm = torch.device("cpu") if dist.get_backend(group) == "gloo" else dev
+    n = torch.tensor([keys.numel()], dtype=torch.int64, device=comm)
     sizes = [torch.zeros_like(n) for _ in range(world)]
     dist.all_gather(sizes, n, group=group)
     m = int(max(int(s.item()) for s in sizes))
     if m == 0:
         e = torch.empty(0, dtype=torch.int64, device=dev)
         return e, e.clone(), e.clone()
-    padded = torch.full((m,), KEY_EMPTY_I64, dtype=torch.int64, device=dev)
-    padded[: keys.numel()] = keys
+    padded = torch.full((m,), KEY_EMPTY_I64, dtype=torch.int64, device=comm)
+    padded[: keys.numel()] = keys.to(comm)
     gathered = [torch.empty_like(padded) for _ in range(world)]
     dist.all_gather(gathered, padded, group=group)
-    union = ops.unique(torch.cat(gathered))
+    union = ops.unique(torch.cat(gathered).to(dev))
     c, f = ops.lookup(union)
+    c, f = c.to(comm), f.to(comm)
     dist.all_reduce(c, op=dist.ReduceOp.SUM, group=group)
     dist.all_reduce(f, op=dist.ReduceOp.MIN, group=group)
-    return union, c, f
+    return union, c.to(dev), f.to(dev)
 
 
 class DeviceOps:

@@ -1,0 +1,123 @@
+"""Parity at BASELINE.json's full size, in the launch configuration bench.py
+times (default TMA kernel, one CTA per SM), plus the multi-rank merge through
+the library's device ops.
+
+* C2 (1e8 records, 1e4 sites, FP32/FP64 50/50, density 1e-6) generated in
+  HBM: the whole GPU table must equal the closed-form aggregate of the
+  planted events (independent of both the oracle and the kernels), and 24
+  random windows of 2048 records must match the CPU oracle entry by entry.
+* 2 ranks (gloo, sharing cuda:0) scan record shards and merge with
+  fpx_table_fetch_device / fpx_keys_unique_device / fpx_table_lookup_device;
+  the merged table must equal one oracle scan of the whole trace.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+import fpxgen
+import oracle
+from _records import DEST, describe_diff, entries_equal, expected_from_injections, table_dict
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+
+def test_c2_full_size_closed_form_and_windows():
+    from paper_conf_hpdc_lilfslg23_b200 import fpx
+
+    n = 100_000_000
+    seed = 0x5EED0000 + 2  # bench.py's C2 seed
+    p = fpxgen.Params(seed=seed, n_records=n, n_sites=10_000, recipe=fpxgen.RECIPE_MIX, p_fp64=0.5)
+    hdr, arena, planes = fpxgen.generate_device(p)
+    inj, writes = fpxgen.plan_injections(p, int(round(1e-6 * n * 32)))
+    fpxgen.apply_device(writes, hdr, arena)
+    with fpx.Handle(0) as h:
+        h.scan_records(hdr, arena, base_index=0, n_records=n, arena_planes=planes)
+        got = h.fetch()
+        assert h.last_status == fpx.OK
+    hdr_host = hdr.cpu().numpy().view(fpxgen.HDR_DTYPE).reshape(-1)
+    exp = expected_from_injections(hdr_host, inj, 0, DEST)
+    assert table_dict(got) == exp
+    assert len(exp) > 1000
+
+    rng = np.random.default_rng(1)
+    with fpx.Handle(0) as h:
+        for w in rng.integers(0, n - 2048, 24):
+            w = int(w)
+            hw = hdr_host[w: w + 2048].copy()
+            lo = int(hw["val_off"][0])
+            hi = int(hw["val_off"][-1]) + 4
+            aw = arena[lo * 32: hi * 32].cpu().numpy().view(np.uint32).reshape(-1, 32)
+            hw["val_off"] -= lo
+            ref = oracle.Table()
+            ref.scan_records(hw, aw, base_index=w)
+            h.reset()
+            d_h = torch.from_numpy(hw.view(np.int32).reshape(-1, 4)).cuda()
+            d_a = torch.from_numpy(aw.view(np.int32).reshape(-1)).cuda()
+            h.scan_records(d_h, d_a, base_index=w)
+            got = h.fetch()
+            assert entries_equal(got, ref.entries()), describe_diff(got, ref.entries())
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _rank(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_hpdc_lilfslg23_b200 import dist as fdist
+    from paper_conf_hpdc_lilfslg23_b200 import fpx
+
+    n = 1_000_003
+    p = fpxgen.Params(seed=5, n_records=n, n_sites=2000, recipe=fpxgen.RECIPE_MIX)
+    hdr, arena, planes = fpxgen.generate_device(p)
+    _, w = fpxgen.plan_injections(p, 2000)
+    fpxgen.apply_device(w, hdr, arena)
+    a, b = fdist.shard_range(n, rank, world)
+    with fpx.Handle(0) as h:
+        h.scan_records(hdr[a:b], arena, base_index=a, arena_planes=planes)
+        k, c, f = fdist.merge_handle(h)
+        q.put((rank, k.cpu().tolist(), c.cpu().tolist(), f.cpu().tolist()))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_two_rank_merge_on_device_ops():
+    import torch.multiprocessing as mp
+
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rank, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for pr in procs:
+        pr.join(timeout=120)
+        assert pr.exitcode == 0
+    n = 1_000_003
+    p = fpxgen.Params(seed=5, n_records=n, n_sites=2000, recipe=fpxgen.RECIPE_MIX)
+    hdr, arena = fpxgen.generate_host(p)
+    _, w = fpxgen.plan_injections(p, 2000)
+    fpxgen.apply_host(w, hdr, arena)
+    t = oracle.Table()
+    t.scan_records(hdr, arena)
+    ref = {}
+    for e in t.entries():
+        k = (int(e["site"]) << 32) | (int(e["fmt"]) << 4) | (int(e["flow"]) << 2) | int(e["kind"])
+        ref[k - (1 << 64) if k >= 1 << 63 else k] = (int(e["count"]), int(e["first_index"]))
+    for rank, k, c, f in res:
+        assert dict(zip(k, zip(c, f))) == ref, rank
+        assert k == sorted(k, key=lambda x: x % (1 << 64))  # ascending uint64 key order
