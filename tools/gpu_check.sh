@@ -34,3 +34,14 @@ if [ "${NCU_TENSOR:-0}" = 1 ]; then
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_scan_tensor -s 3 -c 1 -o $OUT/prof_tensor \
      python bench.py --config c4b --records 1000000000 --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > $OUT/ncu_tensor.log 2>&1; echo "ncu tensor rc=$?"
 fi
+if [ "${NCU_TRAFFIC:-0}" = 1 ]; then
+  # DRAM bytes of the dominant kernel at the full bench configuration (1 replay pass)
+  for cfg in ${TRAFFIC_CONFIGS:-c2}; do
+    timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none \
+      -k regex:k_scan_ -s 4 -c 1 --csv --log-file $OUT/traffic_$cfg.csv \
+      python bench.py --config $cfg --steps 1 --warmup 4 --no-e2e --no-cpu-baseline > $OUT/traffic_$cfg.log 2>&1; echo "traffic $cfg rc=$?"
+  done
+fi
+if [ "${SMOKE:-0}" = 1 ]; then
+  timeout 600 python __graft_entry__.py smoke > $OUT/smoke.log 2>&1; echo "smoke rc=$?"; tail -3 $OUT/smoke.log
+fi
