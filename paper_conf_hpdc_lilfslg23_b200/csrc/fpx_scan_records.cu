@@ -88,23 +88,19 @@ struct RingCfg {
   static constexpr int WARPS = WARPS_, STAGES = STAGES_, PLANES = PLANES_;
 };
 
-// Fast-path item lists of a stage: 4 formats x {full active mask, partial
-// active mask}.  List index = 2 * fmt + partial.
-constexpr int NLISTS = 8;
-
 struct StageMeta {
   uint32_t k;              // records in the tile (0 = no tile)
   uint32_t force;          // tile holds a record that must take the exact path
+  uint32_t n32, n64, n16;  // full-mask fast-path items: FP32 planes, FP64 pairs, FP16x2/BF16x2 planes
+  uint32_t partial;        // bit j: record j has a partial active mask (handled per record)
   uint64_t gidx0;          // global index of the tile's first record
-  uint32_t seg[NLISTS + 1];  // list l = items [seg[l], seg[l+1])
-  uint32_t pad[3];
 };
 
 template <class C>
 struct WarpSmem {
   uint32_t planes[C::STAGES][C::PLANES * 32];  // 128 B per plane
-  uint2 items[C::STAGES][C::PLANES];           // {plane slot, active mask}
-  RecDesc recs[C::STAGES][TILE];
+  uint32_t items[C::STAGES][C::PLANES];        // plane slot (| 1 << 31: BF16x2)
+  RecDesc recs[C::STAGES][TILE];               // meta bits [23:16] slot, [27:24] planes
   StageMeta meta[C::STAGES];
   uint64_t bar[C::STAGES];
 };
@@ -113,31 +109,23 @@ constexpr size_t ring_smem() {
   return sizeof(WarpSmem<C>) * C::WARPS;
 }
 
-// Fast-path item count of a valid, active record.  The items enumerate
-// exactly the planes the mode must look at (DEST: destination words; FLOW:
-// destination + source words), contiguous from plane 0 of the record; an
-// FP64 item is a (lo, hi) pair of planes.
+// Planes of a valid, active record the fast path must look at: DEST the
+// destination words, FLOW destination + source words; contiguous from plane 0
+// of the record.  DIV records (force) and DEST compares need none.
 template <int MODE>
-__device__ __forceinline__ uint32_t record_items(uint32_t meta, bool& force) {
+__device__ __forceinline__ uint32_t record_planes(uint32_t meta, bool& force) {
   const uint32_t op = op_of(meta), fmt = fmt_of(meta), dw = dwords_of(meta), ns = nsrc_of(meta);
   force = op == FPX_OP_DIV;  // DIV0 needs the sources: the exact path reads DIV records itself
   if (force) return 0u;
-  if (MODE == FPX_MODE_DEST) {
-    if (is_compare(op)) return 0u;
-    return fmt == FPX_FP64 ? dw / 2 : dw;
-  }
-  return fmt == FPX_FP64 ? (dw + 2 * ns) / 2 : dw + ns;
-}
-// planes covered by packed item counts (bytes: FP32, FP64 pairs, FP16, BF16)
-__device__ __forceinline__ uint32_t planes_of_items(uint32_t p) {
-  return (p & 0xFFu) + 2u * ((p >> 8) & 0xFFu) + ((p >> 16) & 0xFFu) + (p >> 24);
+  if (MODE == FPX_MODE_DEST) return is_compare(op) ? 0u : dw;
+  return dw + ns * sw_of(fmt);
 }
 
 // Witness updates (no false negatives, exact thresholds in `hit` below).
 //   FP32  a2 = |x| << 1:  subnormal <=> a2 - 2 < 0xFFFFFE;  INF/NaN <=> a2 >= 0xFF000000
 //   FP64  a3 = |hi| | (lo != 0):  subnormal <=> a3 - 1 < 0xFFFFF;  INF/NaN <=> a3 >= 0x7FF00000
 //   FP16 / BF16 per half:  subnormal <=> h - 1 < 0x3FF / 0x7F;  INF/NaN <=> h >= 0x7C00 / 0x7F80
-// `e` masks inactive lanes to zero (zero is clean in every format).
+// Inactive lanes are masked to zero (zero is clean in every format).
 struct Witness {
   uint32_t mn32 = 0xFFFFFFFFu, mx32 = 0u, mn64 = 0xFFFFFFFFu, mx64 = 0u;
   uint32_t mn16 = 0xFFFFFFFFu, mx16 = 0u, mnb = 0xFFFFFFFFu, mxb = 0u;
@@ -173,6 +161,7 @@ __global__ void __launch_bounds__(C::WARPS * 32, 1)
 k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __restrict__ arena,
                    uint64_t arena_planes, uint64_t base_index, uint64_t recs_per_warp, const TableView tv) {
   constexpr int STAGES = C::STAGES, PLANES = C::PLANES;
+  static_assert(PLANES <= 255, "plane slots are 8-bit");
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   WarpSmem<C>& sm = reinterpret_cast<WarpSmem<C>*>(smem_raw)[warp];
@@ -207,63 +196,59 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const bool ok = inrange && record_valid<MODE>(h, arena_planes);
     const uint32_t mask = ok ? h.y : 0u;
     bool force = false;
+    const uint32_t c_all = (ok && mask != 0u) ? record_planes<MODE>(h.z, force) : 0u;
     const uint32_t fmt = fmt_of(h.z);
-    const uint32_t ni = (ok && mask != 0u) ? record_items<MODE>(h.z, force) : 0u;
-    const bool part = mask != FULL;
-    // two packed scans (full-mask / partial-mask records; byte = format)
-    const uint32_t cf = part ? 0u : ni << (8 * fmt), cp = part ? ni << (8 * fmt) : 0u;
-    uint32_t sf = cf, sp = cp;
+    const bool full = mask == FULL;
+    // one packed scan: [31:24] planes, [23:16] FP16x2+BF16x2 items, [15:8]
+    // FP64 pairs, [7:0] FP32 items (items of full-mask records only); planes
+    // may wrap past the tile, item fields cannot overflow (<= 4 per record)
+    const uint32_t nit = !full ? 0u : (fmt == FPX_FP64 ? c_all >> 1 : c_all);
+    const uint32_t cnt = (c_all << 24) | (nit << (8 * (fmt >= 2u ? 2u : fmt)));
+    uint32_t sc = cnt;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t tf = __shfl_up_sync(FULL, sf, o), tp = __shfl_up_sync(FULL, sp, o);
-      if (lane >= o) { sf += tf; sp += tp; }
+      const uint32_t t = __shfl_up_sync(FULL, sc, o);
+      if (lane >= o) sc += t;
     }
-    const uint32_t incl_planes = planes_of_items(sf) + planes_of_items(sp);
     // the tile = leading records whose planes fit the stage (>= 1 record)
-    const uint32_t k = __popc(__ballot_sync(FULL, inrange && incl_planes <= (uint32_t)PLANES));
+    const uint32_t fits = __ballot_sync(FULL, inrange && (sc >> 24) <= (uint32_t)PLANES);
+    const uint32_t k = ~fits == 0u ? 32u : (uint32_t)(__ffs(~fits) - 1);
     const bool in_tile = (uint32_t)lane < k;
     const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
     if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
-    const uint32_t my_planes = planes_of_items(cf + cp);
-    const uint32_t c = in_tile ? my_planes : 0u;
-    const uint32_t slot = incl_planes - my_planes;
-    const uint32_t tf = __shfl_sync(FULL, sf, k - 1), tp = __shfl_sync(FULL, sp, k - 1);
-    const uint32_t total = planes_of_items(tf) + planes_of_items(tp);
-    const bool force_any = __any_sync(FULL, in_tile && force);
+    const uint32_t c = in_tile ? c_all : 0u;
+    const uint32_t ex = sc - cnt;
+    const uint32_t slot = ex >> 24;
+    const uint32_t tot = __shfl_sync(FULL, sc, k - 1);
+    const uint32_t total = tot >> 24;
+    const uint32_t n32 = tot & 0xFFu, n64 = (tot >> 8) & 0xFFu, n16 = (tot >> 16) & 0xFFu;
+    const uint32_t force_any = __ballot_sync(FULL, in_tile && force);
+    const uint32_t partial = __ballot_sync(FULL, in_tile && c != 0u && !full);
     // the ring slot may still be read by the previous consume of this stage:
     // order those generic reads before the async-proxy writes below
     __syncwarp();
     fence_proxy_async_smem();
-    sm.recs[s][lane] = in_tile ? RecDesc{h.w, mask, h.z, h.x} : RecDesc{0u, 0u, 0u, 0u};
-    // list l = 2*fmt + partial starts after all lists of lower formats
-    const uint32_t tot_f = tf + tp;  // per-format item totals (packed)
-    if (in_tile && ni != 0u) {
-      const uint32_t below = (0x00000000u + (fmt > 0 ? (tot_f & 0xFFu) : 0u) + (fmt > 1 ? ((tot_f >> 8) & 0xFFu) : 0u) +
-                              (fmt > 2 ? ((tot_f >> 16) & 0xFFu) : 0u));
-      const uint32_t at = below + (part ? ((tf >> (8 * fmt)) & 0xFFu) : 0u) +
-                          (((part ? sp - cp : sf - cf) >> (8 * fmt)) & 0xFFu);
-      const uint32_t step = fmt == FPX_FP64 ? 2u : 1u;
-      for (uint32_t q = 0; q < ni; ++q) sm.items[s][at + q] = make_uint2(slot + q * step, mask);
+    sm.recs[s][lane] = in_tile ? RecDesc{h.w, mask, h.z | (slot << 16) | (c << 24), h.x} : RecDesc{0u, 0u, 0u, 0u};
+    if (in_tile && nit != 0u) {
+      const uint32_t fl = fmt >= 2u ? 2u : fmt;
+      const uint32_t at = (fl == 0u ? 0u : fl == 1u ? n32 : n32 + n64) + ((ex >> (8 * fl)) & 0xFFu);
+      const uint32_t tag = fmt == FPX_BF16 ? 0x80000000u : 0u;
+      for (uint32_t q = 0; q < nit; ++q) sm.items[s][at + q] = (slot + (fmt == FPX_FP64 ? 2u * q : q)) | tag;
     }
     if (lane == 0) {
       m.k = k;
-      m.force = force_any ? 1u : 0u;
+      m.force = force_any;
+      m.n32 = n32;
+      m.n64 = n64;
+      m.n16 = n16;
+      m.partial = partial;
       m.gidx0 = base_index + cursor;
-      uint32_t acc = 0;
-#pragma unroll
-      for (int f = 0; f < 4; ++f) {
-        m.seg[2 * f] = acc;
-        acc += (tf >> (8 * f)) & 0xFFu;
-        m.seg[2 * f + 1] = acc;
-        acc += (tp >> (8 * f)) & 0xFFu;
-      }
-      m.seg[NLISTS] = acc;
     }
-    // runs of arena-adjacent records -> one bulk copy each
+    // runs of arena-adjacent planes -> one bulk copy each (a record with no
+    // needed planes and no arena footprint does not break a run)
     const uint32_t a = h.w;
     const uint32_t prev_end = __shfl_up_sync(FULL, a + c, 1);
-    const uint32_t prev_c = __shfl_up_sync(FULL, c, 1);
-    const bool head = c != 0u && (lane == 0 || prev_c == 0u || prev_end != a);
+    const bool head = c != 0u && (lane == 0 || prev_end != a);
     const uint32_t heads = __ballot_sync(FULL, head);
     const uint32_t above = lane == 31 ? 0u : heads & (0xFFFFFFFFu << (lane + 1));  // heads above this lane
     const uint32_t next = above ? (uint32_t)(__ffs(above) - 1) : 32u;
@@ -294,32 +279,34 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 
     // ---- fast path over the staged planes --------------------------------
     const uint32_t* __restrict__ pl = sm.planes[s] + lane;
-    const uint2* __restrict__ it = sm.items[s];
-    uint32_t seg[NLISTS + 1];
-#pragma unroll
-    for (int l = 0; l <= NLISTS; ++l) seg[l] = m.seg[l];
+    const uint32_t* __restrict__ it = sm.items[s];
+    const uint32_t n32 = m.n32, e64 = n32 + m.n64, e16 = e64 + m.n16;
     Witness w;
 #pragma unroll 4
-    for (uint32_t q = seg[0]; q < seg[1]; ++q) w.fp32(pl[it[q].x * 32]);
-    for (uint32_t q = seg[1]; q < seg[2]; ++q) {
-      const uint2 t = it[q];
-      w.fp32(pl[t.x * 32] & lane_ext(t.y, lane));
-    }
+    for (uint32_t q = 0; q < n32; ++q) w.fp32(pl[it[q] * 32]);
 #pragma unroll 4
-    for (uint32_t q = seg[2]; q < seg[3]; ++q) {
-      const uint32_t t = it[q].x * 32;
+    for (uint32_t q = n32; q < e64; ++q) {
+      const uint32_t t = it[q] * 32;
       w.fp64(pl[t], pl[t + 32]);
     }
-    for (uint32_t q = seg[3]; q < seg[4]; ++q) {
-      const uint2 t = it[q];
-      const uint32_t e = lane_ext(t.y, lane);
-      w.fp64(pl[t.x * 32] & e, pl[t.x * 32 + 32] & e);
+#pragma unroll 2
+    for (uint32_t q = e64; q < e16; ++q) {
+      const uint32_t t = it[q];
+      w.half2(pl[(t & 0xFFu) * 32], (t >> 31) != 0u);
     }
-    for (uint32_t q = seg[4]; q < seg[8]; ++q) {
-      const uint2 t = it[q];
-      const bool partial = (q >= seg[5] && q < seg[6]) || q >= seg[7];
-      const uint32_t e = partial ? lane_ext(t.y, lane) : 0xFFFFFFFFu;
-      w.half2(pl[t.x * 32] & e, q >= seg[6]);
+    // partial-mask records, one at a time, inactive lanes masked to zero
+    for (uint32_t pm = m.partial; pm != 0u; pm &= pm - 1u) {
+      const RecDesc d = sm.recs[s][__ffs(pm) - 1];
+      const uint32_t e = lane_ext(d.mask, lane);
+      const uint32_t fmt = fmt_of(d.meta), slot = (d.meta >> 16) & 0xFFu, c = d.meta >> 24;
+      const uint32_t* p = pl + slot * 32;
+      if (fmt == FPX_FP32) {
+        for (uint32_t q = 0; q < c; ++q) w.fp32(p[q * 32] & e);
+      } else if (fmt == FPX_FP64) {
+        for (uint32_t q = 0; q < c; q += 2) w.fp64(p[q * 32] & e, p[q * 32 + 32] & e);
+      } else {
+        for (uint32_t q = 0; q < c; ++q) w.half2(p[q * 32] & e, fmt == FPX_BF16);
+      }
     }
     if (__any_sync(FULL, w.hit()) || m.force) exact_tile<MODE>(sm.recs[s], lane_base, lane, m.gidx0, tv);
   }
