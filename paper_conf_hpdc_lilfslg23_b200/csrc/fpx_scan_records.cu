@@ -58,8 +58,19 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
       : "memory");
   return ok != 0;
 }
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+// Bounded wait: the copies of a stage always complete unless the byte count
+// promised by expect_tx and the bytes issued disagree (an internal bug); a
+// watchdog turns such a deadlock into a launch error instead of a hang.
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  if (mbar_try_wait(bar, parity)) return;
+  const uint64_t t0 = globaltimer_ns();
   while (!mbar_try_wait(bar, parity)) {
+    if (globaltimer_ns() - t0 > 4000000000ull) __trap();
   }
 }
 // global -> shared bulk copy (TMA), completion counted in bytes on `bar`;
@@ -244,11 +255,12 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       m.partial = partial;
       m.gidx0 = base_index + cursor;
     }
-    // runs of arena-adjacent planes -> one bulk copy each (a record with no
-    // needed planes and no arena footprint does not break a run)
+    // runs of arena-adjacent records -> one bulk copy each; a record with no
+    // needed planes ends a run (its own footprint is unknown here)
     const uint32_t a = h.w;
     const uint32_t prev_end = __shfl_up_sync(FULL, a + c, 1);
-    const bool head = c != 0u && (lane == 0 || prev_end != a);
+    const uint32_t prev_c = __shfl_up_sync(FULL, c, 1);
+    const bool head = c != 0u && (lane == 0 || prev_c == 0u || prev_end != a);
     const uint32_t heads = __ballot_sync(FULL, head);
     const uint32_t above = lane == 31 ? 0u : heads & (0xFFFFFFFFu << (lane + 1));  // heads above this lane
     const uint32_t next = above ? (uint32_t)(__ffs(above) - 1) : 32u;

@@ -8,7 +8,7 @@ nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,memory.total,power.limit --f
 nproc > $OUT/host.txt; lscpu | grep -E "Model name|^CPU\(s\)" >> $OUT/host.txt
 python __graft_entry__.py build > $OUT/build.log 2>&1 || { echo BUILD FAILED; tail -50 $OUT/build.log; exit 1; }
 if [ "${TESTS:-1}" = 1 ]; then
-  timeout 1200 python -m pytest tests -m gpu -x -q ${PYTEST_ARGS:-} > $OUT/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> $OUT/pytest_gpu.log
+  timeout 900 python -m pytest tests -m gpu -x -q --timeout 240 ${PYTEST_ARGS:-} > $OUT/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> $OUT/pytest_gpu.log
   tail -30 $OUT/pytest_gpu.log
 fi
 if [ "${BENCH:-1}" = 1 ]; then
