@@ -99,19 +99,23 @@ struct RingCfg {
   static constexpr int WARPS = WARPS_, STAGES = STAGES_, PLANES = PLANES_;
 };
 
+// Fast-path item lists of a stage: 4 formats x {full, partial active mask}.
+// list l = 2 * fmt + partial.
+constexpr int NLISTS = 8;
+
 struct StageMeta {
-  uint32_t k;              // records in the tile (0 = no tile)
-  uint32_t force;          // tile holds a record that must take the exact path
-  uint32_t n32, n64, n16;  // full-mask fast-path items: FP32 planes, FP64 pairs, FP16x2/BF16x2 planes
-  uint32_t partial;        // bit j: record j has a partial active mask (handled per record)
-  uint64_t gidx0;          // global index of the tile's first record
+  uint32_t k;                // records in the tile (0 = no tile)
+  uint32_t force;            // tile holds a record that must take the exact path
+  uint64_t gidx0;            // global index of the tile's first record
+  uint32_t seg[NLISTS + 1];  // list l = items [seg[l], seg[l+1])
+  uint32_t pad[3];
 };
 
 template <class C>
 struct WarpSmem {
   uint32_t planes[C::STAGES][C::PLANES * 32];  // 128 B per plane
-  uint32_t items[C::STAGES][C::PLANES];        // plane slot (| 1 << 31: BF16x2)
-  RecDesc recs[C::STAGES][TILE];               // meta bits [23:16] slot, [27:24] planes
+  uint2 items[C::STAGES][C::PLANES];           // {plane slot, active mask}
+  RecDesc recs[C::STAGES][TILE];
   StageMeta meta[C::STAGES];
   uint64_t bar[C::STAGES];
 };
@@ -120,23 +124,31 @@ constexpr size_t ring_smem() {
   return sizeof(WarpSmem<C>) * C::WARPS;
 }
 
-// Planes of a valid, active record the fast path must look at: DEST the
-// destination words, FLOW destination + source words; contiguous from plane 0
-// of the record.  DIV records (force) and DEST compares need none.
+// Fast-path items of a valid, active record: they enumerate exactly the planes
+// the mode must look at (DEST: destination words; FLOW: destination + source
+// words), contiguous from plane 0 of the record; an FP64 item is a (lo, hi)
+// pair of planes.  DIV records (force) and DEST compares have none.
 template <int MODE>
-__device__ __forceinline__ uint32_t record_planes(uint32_t meta, bool& force) {
+__device__ __forceinline__ uint32_t record_items(uint32_t meta, bool& force) {
   const uint32_t op = op_of(meta), fmt = fmt_of(meta), dw = dwords_of(meta), ns = nsrc_of(meta);
   force = op == FPX_OP_DIV;  // DIV0 needs the sources: the exact path reads DIV records itself
   if (force) return 0u;
-  if (MODE == FPX_MODE_DEST) return is_compare(op) ? 0u : dw;
-  return dw + ns * sw_of(fmt);
+  uint32_t p;
+  if (MODE == FPX_MODE_DEST) p = is_compare(op) ? 0u : dw;
+  else p = dw + ns * sw_of(fmt);
+  return fmt == FPX_FP64 ? p >> 1 : p;
+}
+// planes covered by packed item counts (bytes: FP32, FP64 pairs, FP16, BF16;
+// each byte <= 128 so the byte sum cannot overflow)
+__device__ __forceinline__ uint32_t planes_of_items(uint32_t p) {
+  return ((p * 0x01010101u) >> 24) + ((p >> 8) & 0xFFu);
 }
 
-// Witness updates (no false negatives, exact thresholds in `hit` below).
+// Witnesses of one 32-bit word (no false negatives; exact thresholds in hit()):
 //   FP32  a2 = |x| << 1:  subnormal <=> a2 - 2 < 0xFFFFFE;  INF/NaN <=> a2 >= 0xFF000000
 //   FP64  a3 = |hi| | (lo != 0):  subnormal <=> a3 - 1 < 0xFFFFF;  INF/NaN <=> a3 >= 0x7FF00000
 //   FP16 / BF16 per half:  subnormal <=> h - 1 < 0x3FF / 0x7F;  INF/NaN <=> h >= 0x7C00 / 0x7F80
-// Inactive lanes are masked to zero (zero is clean in every format).
+// Inactive lanes are masked to zero first (zero is clean in every format).
 struct Witness {
   uint32_t mn32 = 0xFFFFFFFFu, mx32 = 0u, mn64 = 0xFFFFFFFFu, mx64 = 0u;
   uint32_t mn16 = 0xFFFFFFFFu, mx16 = 0u, mnb = 0xFFFFFFFFu, mxb = 0u;
@@ -150,10 +162,11 @@ struct Witness {
     mn64 = min(mn64, a3 - 1u);
     mx64 = max(mx64, a3);
   }
-  __device__ __forceinline__ void half2(uint32_t x, bool bf) {
+  template <bool BF>
+  __device__ __forceinline__ void half2(uint32_t x) {
     x &= 0x7FFF7FFFu;
     const uint32_t l = x & 0xFFFFu, h = x >> 16;
-    if (bf) {
+    if (BF) {
       mnb = min(mnb, min(l - 1u, h - 1u));
       mxb = max(mxb, max(l, h));
     } else {
@@ -167,12 +180,72 @@ struct Witness {
   }
 };
 
+// 128-bit shared load at a byte address.
+__device__ __forceinline__ uint4 lds128(uint32_t addr) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ uint2 lds64(uint32_t addr) {
+  uint2 v;
+  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(addr));
+  return v;
+}
+// Per-value activity masks of lanes 4q .. 4q+3 (all ones = active).
+__device__ __forceinline__ uint4 quad_ext(uint32_t mask, uint32_t q) {
+  const uint32_t m = mask >> (4 * q);
+  return make_uint4((uint32_t)((int32_t)(m << 31) >> 31), (uint32_t)((int32_t)(m << 30) >> 31),
+                    (uint32_t)((int32_t)(m << 29) >> 31), (uint32_t)((int32_t)(m << 28) >> 31));
+}
+__device__ __forceinline__ uint4 and4(uint4 a, uint4 b) { return make_uint4(a.x & b.x, a.y & b.y, a.z & b.z, a.w & b.w); }
+
+// Consume one item list with the lane-quad layout: thread (g = lane / 8,
+// q = lane % 8) reads words 4q..4q+3 (lanes 4q..4q+3 of the instrumented
+// warp) of item i + g, so one warp step covers four items with one 128-bit
+// shared load per thread (two for an FP64 pair).
+template <uint32_t FMT, bool PARTIAL>
+__device__ __forceinline__ void consume_list(Witness& w, uint32_t b, uint32_t e, uint32_t items_addr,
+                                             uint32_t planes_addr, uint32_t g, uint32_t q) {
+#pragma unroll 2
+  for (uint32_t i = b + g; i < e; i += 4) {
+    const uint2 it = lds64(items_addr + i * 8);
+    const uint32_t a = planes_addr + it.x * 128 + q * 16;
+    uint4 x = lds128(a);
+    uint4 mk = make_uint4(~0u, ~0u, ~0u, ~0u);
+    if (PARTIAL) mk = quad_ext(it.y, q);
+    if (FMT == FPX_FP64) {
+      uint4 hi = lds128(a + 128);
+      if (PARTIAL) {
+        x = and4(x, mk);
+        hi = and4(hi, mk);
+      }
+      w.fp64(x.x, hi.x);
+      w.fp64(x.y, hi.y);
+      w.fp64(x.z, hi.z);
+      w.fp64(x.w, hi.w);
+    } else {
+      if (PARTIAL) x = and4(x, mk);
+      if (FMT == FPX_FP32) {
+        w.fp32(x.x);
+        w.fp32(x.y);
+        w.fp32(x.z);
+        w.fp32(x.w);
+      } else {
+        w.half2<FMT == FPX_BF16>(x.x);
+        w.half2<FMT == FPX_BF16>(x.y);
+        w.half2<FMT == FPX_BF16>(x.z);
+        w.half2<FMT == FPX_BF16>(x.w);
+      }
+    }
+  }
+}
+
 template <int MODE, class C>
 __global__ void __launch_bounds__(C::WARPS * 32, 1)
 k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __restrict__ arena,
                    uint64_t arena_planes, uint64_t base_index, uint64_t recs_per_warp, const TableView tv) {
   constexpr int STAGES = C::STAGES, PLANES = C::PLANES;
-  static_assert(PLANES <= 255, "plane slots are 8-bit");
+  static_assert(PLANES <= 64, "stage sizes keep the byte fields of the packed scan exact");
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   WarpSmem<C>& sm = reinterpret_cast<WarpSmem<C>*>(smem_raw)[warp];
@@ -182,6 +255,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   const uint64_t end = min(n, start + recs_per_warp);
   const uint32_t* __restrict__ lane_base = arena + lane;
   const uint64_t policy = policy_evict_first();
+  const uint32_t g = (uint32_t)lane >> 3, q = (uint32_t)lane & 7u;
 
   if (lane == 0) {
 #pragma unroll
@@ -207,52 +281,55 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const bool ok = inrange && record_valid<MODE>(h, arena_planes);
     const uint32_t mask = ok ? h.y : 0u;
     bool force = false;
-    const uint32_t c_all = (ok && mask != 0u) ? record_planes<MODE>(h.z, force) : 0u;
     const uint32_t fmt = fmt_of(h.z);
-    const bool full = mask == FULL;
-    // one packed scan: [31:24] planes, [23:16] FP16x2+BF16x2 items, [15:8]
-    // FP64 pairs, [7:0] FP32 items (items of full-mask records only); planes
-    // may wrap past the tile, item fields cannot overflow (<= 4 per record)
-    const uint32_t nit = !full ? 0u : (fmt == FPX_FP64 ? c_all >> 1 : c_all);
-    const uint32_t cnt = (c_all << 24) | (nit << (8 * (fmt >= 2u ? 2u : fmt)));
-    uint32_t sc = cnt;
+    const uint32_t ni = (ok && mask != 0u) ? record_items<MODE>(h.z, force) : 0u;
+    const bool part = mask != FULL;
+    // two packed scans (full / partial active mask; byte = format).  Bytes
+    // stay <= 128 over the warp, so no field overflows into the next.
+    const uint32_t c8 = ni << (8 * fmt);
+    const uint32_t cf = part ? 0u : c8, cp = part ? c8 : 0u;
+    uint32_t sf = cf, sp = cp;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t t = __shfl_up_sync(FULL, sc, o);
-      if (lane >= o) sc += t;
+      const uint32_t tf = __shfl_up_sync(FULL, sf, o), tp = __shfl_up_sync(FULL, sp, o);
+      if (lane >= o) { sf += tf; sp += tp; }
     }
+    const uint32_t incl_planes = planes_of_items(sf) + planes_of_items(sp);
     // the tile = leading records whose planes fit the stage (>= 1 record)
-    const uint32_t fits = __ballot_sync(FULL, inrange && (sc >> 24) <= (uint32_t)PLANES);
+    const uint32_t fits = __ballot_sync(FULL, inrange && incl_planes <= (uint32_t)PLANES);
     const uint32_t k = ~fits == 0u ? 32u : (uint32_t)(__ffs(~fits) - 1);
     const bool in_tile = (uint32_t)lane < k;
     const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
     if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
-    const uint32_t c = in_tile ? c_all : 0u;
-    const uint32_t ex = sc - cnt;
-    const uint32_t slot = ex >> 24;
-    const uint32_t tot = __shfl_sync(FULL, sc, k - 1);
-    const uint32_t total = tot >> 24;
-    const uint32_t n32 = tot & 0xFFu, n64 = (tot >> 8) & 0xFFu, n16 = (tot >> 16) & 0xFFu;
+    const uint32_t my_planes = planes_of_items(c8);
+    const uint32_t c = in_tile ? my_planes : 0u;
+    const uint32_t slot = incl_planes - my_planes;
+    const uint32_t tf = __shfl_sync(FULL, sf, k - 1), tp = __shfl_sync(FULL, sp, k - 1);
+    const uint32_t total = planes_of_items(tf) + planes_of_items(tp);
     const uint32_t force_any = __ballot_sync(FULL, in_tile && force);
-    const uint32_t partial = __ballot_sync(FULL, in_tile && c != 0u && !full);
     // the ring slot may still be read by the previous consume of this stage:
     // order those generic reads before the async-proxy writes below
     __syncwarp();
     fence_proxy_async_smem();
-    sm.recs[s][lane] = in_tile ? RecDesc{h.w, mask, h.z | (slot << 16) | (c << 24), h.x} : RecDesc{0u, 0u, 0u, 0u};
-    if (in_tile && nit != 0u) {
-      const uint32_t fl = fmt >= 2u ? 2u : fmt;
-      const uint32_t at = (fl == 0u ? 0u : fl == 1u ? n32 : n32 + n64) + ((ex >> (8 * fl)) & 0xFFu);
-      const uint32_t tag = fmt == FPX_BF16 ? 0x80000000u : 0u;
-      for (uint32_t q = 0; q < nit; ++q) sm.items[s][at + q] = (slot + (fmt == FPX_FP64 ? 2u * q : q)) | tag;
+    sm.recs[s][lane] = in_tile ? RecDesc{h.w, mask, h.z, h.x} : RecDesc{0u, 0u, 0u, 0u};
+    // list l = 2 * fmt + partial; lists of lower formats come first
+    const uint32_t tot_f = tf + tp;  // packed per-format item totals (<= 128 each)
+    if (in_tile && ni != 0u) {
+      const uint32_t below = ((tot_f << (32 - 8 * fmt)) * 0x01010101u) >> 24;  // byte sum of formats < fmt
+      const uint32_t at = (fmt == 0u ? 0u : below) + (part ? ((tf >> (8 * fmt)) & 0xFFu) : 0u) +
+                          (((part ? sp - cp : sf - cf) >> (8 * fmt)) & 0xFFu);
+      const uint32_t step = fmt == FPX_FP64 ? 2u : 1u;
+      for (uint32_t j = 0; j < ni; ++j) sm.items[s][at + j] = make_uint2(slot + j * step, mask);
+    }
+    if (lane <= NLISTS) {  // seg[l] = items of lists < l
+      const uint32_t f = (uint32_t)lane >> 1;
+      const uint32_t lower = f == 0u ? 0u : (f >= 4u ? (tot_f * 0x01010101u) >> 24
+                                                     : ((tot_f << (32 - 8 * f)) * 0x01010101u) >> 24);
+      m.seg[lane] = lower + ((lane & 1) && f < 4u ? ((tf >> (8 * f)) & 0xFFu) : 0u);
     }
     if (lane == 0) {
       m.k = k;
       m.force = force_any;
-      m.n32 = n32;
-      m.n64 = n64;
-      m.n16 = n16;
-      m.partial = partial;
       m.gidx0 = base_index + cursor;
     }
     // runs of arena-adjacent records -> one bulk copy each; a record with no
@@ -284,41 +361,25 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const int s = (int)(i % STAGES);
     produce((int)((i + STAGES - 1) % STAGES));
     const StageMeta& m = sm.meta[s];
-    const uint32_t k = m.k;
-    if (k == 0u) break;
+    if (m.k == 0u) break;
     mbar_wait(&sm.bar[s], (phase >> s) & 1u);
     phase ^= 1u << s;
 
-    // ---- fast path over the staged planes --------------------------------
-    const uint32_t* __restrict__ pl = sm.planes[s] + lane;
-    const uint32_t* __restrict__ it = sm.items[s];
-    const uint32_t n32 = m.n32, e64 = n32 + m.n64, e16 = e64 + m.n16;
+    // ---- fast path over the staged planes (lane-quad layout) --------------
+    const uint32_t ia = smem_u32(sm.items[s]), pa = smem_u32(sm.planes[s]);
+    uint32_t seg[NLISTS + 1];
+#pragma unroll
+    for (int l = 0; l <= NLISTS; ++l) seg[l] = m.seg[l];
     Witness w;
-#pragma unroll 4
-    for (uint32_t q = 0; q < n32; ++q) w.fp32(pl[it[q] * 32]);
-#pragma unroll 4
-    for (uint32_t q = n32; q < e64; ++q) {
-      const uint32_t t = it[q] * 32;
-      w.fp64(pl[t], pl[t + 32]);
-    }
-#pragma unroll 2
-    for (uint32_t q = e64; q < e16; ++q) {
-      const uint32_t t = it[q];
-      w.half2(pl[(t & 0xFFu) * 32], (t >> 31) != 0u);
-    }
-    // partial-mask records, one at a time, inactive lanes masked to zero
-    for (uint32_t pm = m.partial; pm != 0u; pm &= pm - 1u) {
-      const RecDesc d = sm.recs[s][__ffs(pm) - 1];
-      const uint32_t e = lane_ext(d.mask, lane);
-      const uint32_t fmt = fmt_of(d.meta), slot = (d.meta >> 16) & 0xFFu, c = d.meta >> 24;
-      const uint32_t* p = pl + slot * 32;
-      if (fmt == FPX_FP32) {
-        for (uint32_t q = 0; q < c; ++q) w.fp32(p[q * 32] & e);
-      } else if (fmt == FPX_FP64) {
-        for (uint32_t q = 0; q < c; q += 2) w.fp64(p[q * 32] & e, p[q * 32 + 32] & e);
-      } else {
-        for (uint32_t q = 0; q < c; ++q) w.half2(p[q * 32] & e, fmt == FPX_BF16);
-      }
+    consume_list<FPX_FP32, false>(w, seg[0], seg[1], ia, pa, g, q);
+    consume_list<FPX_FP32, true>(w, seg[1], seg[2], ia, pa, g, q);
+    consume_list<FPX_FP64, false>(w, seg[2], seg[3], ia, pa, g, q);
+    consume_list<FPX_FP64, true>(w, seg[3], seg[4], ia, pa, g, q);
+    if (seg[4] != seg[8]) {
+      consume_list<FPX_FP16, false>(w, seg[4], seg[5], ia, pa, g, q);
+      consume_list<FPX_FP16, true>(w, seg[5], seg[6], ia, pa, g, q);
+      consume_list<FPX_BF16, false>(w, seg[6], seg[7], ia, pa, g, q);
+      consume_list<FPX_BF16, true>(w, seg[7], seg[8], ia, pa, g, q);
     }
     if (__any_sync(FULL, w.hit()) || m.force) exact_tile<MODE>(sm.recs[s], lane_base, lane, m.gidx0, tv);
   }
