@@ -124,19 +124,29 @@ constexpr size_t ring_smem() {
   return sizeof(WarpSmem<C>) * C::WARPS;
 }
 
-// Fast-path items of a valid, active record: they enumerate exactly the planes
-// the mode must look at (DEST: destination words; FLOW: destination + source
-// words), contiguous from plane 0 of the record; an FP64 item is a (lo, hi)
-// pair of planes.  DIV records (force) and DEST compares have none.
+// Header decode for the fast path, branch-free: validity (the contract of
+// include/fpx.h, same rules as rec::record_valid), the number of fast-path
+// items (they enumerate exactly the planes the mode must look at — DEST: the
+// destination words; FLOW: destination + source words — contiguous from plane
+// 0 of the record; an FP64 item is a (lo, hi) pair), and `force` for DIV
+// records, whose DIV0 rule needs the sources: the exact path reads them.
 template <int MODE>
-__device__ __forceinline__ uint32_t record_items(uint32_t meta, bool& force) {
-  const uint32_t op = op_of(meta), fmt = fmt_of(meta), dw = dwords_of(meta), ns = nsrc_of(meta);
-  force = op == FPX_OP_DIV;  // DIV0 needs the sources: the exact path reads DIV records itself
-  if (force) return 0u;
-  uint32_t p;
-  if (MODE == FPX_MODE_DEST) p = is_compare(op) ? 0u : dw;
-  else p = dw + ns * sw_of(fmt);
-  return fmt == FPX_FP64 ? p >> 1 : p;
+__device__ __forceinline__ uint32_t decode_items(const uint4 h, uint64_t arena_planes, bool inrange, bool& ok,
+                                                 bool& force) {
+  const uint32_t meta = h.z;
+  const uint32_t op = meta & 0xFFu, fmt = (meta >> 8) & 3u, ns = (meta >> 10) & 3u, dw = (meta >> 12) & 7u;
+  const uint32_t is64 = fmt == FPX_FP64 ? 1u : 0u;
+  const uint32_t all_planes = dw + (ns << is64);
+  bool v = inrange & (h.x != FPX_SITE_INVALID) & (meta < 0x8000u) & (op < (uint32_t)FPX_OP_COUNT) & (dw <= 4u) &
+           !((is64 != 0u) & ((dw & 1u) != 0u));
+  v &= (uint64_t)h.w + all_planes <= arena_planes;
+  if (MODE == FPX_MODE_FLOW) v &= (fmt <= 1u) & ((dw == 0u) | (dw == 1u + is64));
+  ok = v;
+  const bool live = v & (h.y != 0u);
+  force = live & (op == FPX_OP_DIV);
+  uint32_t p = all_planes;
+  if (MODE == FPX_MODE_DEST) p = ((0x5800u >> (op & 31u)) & 1u) ? 0u : dw;  // FSET / FSETP / DSETP: no dest kind
+  return (live & !force) ? (p >> is64) : 0u;
 }
 // planes covered by packed item counts (bytes: FP32, FP64 pairs, FP16, BF16;
 // each byte <= 128 so the byte sum cannot overflow)
@@ -278,11 +288,10 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       return;
     }
     const bool inrange = cursor + lane < end;
-    const bool ok = inrange && record_valid<MODE>(h, arena_planes);
+    bool ok, force;
+    const uint32_t ni = decode_items<MODE>(h, arena_planes, inrange, ok, force);
     const uint32_t mask = ok ? h.y : 0u;
-    bool force = false;
     const uint32_t fmt = fmt_of(h.z);
-    const uint32_t ni = (ok && mask != 0u) ? record_items<MODE>(h.z, force) : 0u;
     const bool part = mask != FULL;
     // two packed scans (full / partial active mask; byte = format).  Bytes
     // stay <= 128 over the warp, so no field overflows into the next.
@@ -319,7 +328,9 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       const uint32_t at = (fmt == 0u ? 0u : below) + (part ? ((tf >> (8 * fmt)) & 0xFFu) : 0u) +
                           (((part ? sp - cp : sf - cf) >> (8 * fmt)) & 0xFFu);
       const uint32_t step = fmt == FPX_FP64 ? 2u : 1u;
-      for (uint32_t j = 0; j < ni; ++j) sm.items[s][at + j] = make_uint2(slot + j * step, mask);
+#pragma unroll
+      for (uint32_t j = 0; j < 4; ++j)  // ni <= 4
+        if (j < ni) sm.items[s][at + j] = make_uint2(slot + j * step, mask);
     }
     if (lane <= NLISTS) {  // seg[l] = items of lists < l
       const uint32_t f = (uint32_t)lane >> 1;
