@@ -148,6 +148,11 @@ __device__ __forceinline__ uint32_t decode_items(const uint4 h, uint64_t arena_p
   if (MODE == FPX_MODE_DEST) p = ((0x5800u >> (op & 31u)) & 1u) ? 0u : dw;  // FSET / FSETP / DSETP: no dest kind
   return (live & !force) ? (p >> is64) : 0u;
 }
+// arena planes a record occupies (destination + all sources)
+__device__ __forceinline__ uint32_t footprint(uint32_t meta) {
+  return dwords_of(meta) + (nsrc_of(meta) << (fmt_of(meta) == FPX_FP64 ? 1u : 0u));
+}
+
 // planes covered by packed item counts (bytes: FP32, FP64 pairs, FP16, BF16;
 // each byte <= 128 so the byte sum cannot overflow)
 __device__ __forceinline__ uint32_t planes_of_items(uint32_t p) {
@@ -343,12 +348,16 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       m.force = force_any;
       m.gidx0 = base_index + cursor;
     }
-    // runs of arena-adjacent records -> one bulk copy each; a record with no
-    // needed planes ends a run (its own footprint is unknown here)
+    // runs of arena-adjacent needed planes -> one bulk copy each.  Records
+    // with no arena footprint are transparent; a record whose needed planes
+    // stop before the end of its footprint (DEST with sources) ends a run.
     const uint32_t a = h.w;
-    const uint32_t prev_end = __shfl_up_sync(FULL, a + c, 1);
-    const uint32_t prev_c = __shfl_up_sync(FULL, c, 1);
-    const bool head = c != 0u && (lane == 0 || prev_c == 0u || prev_end != a);
+    const uint32_t foot = in_tile ? footprint(h.z) : 0u;
+    const uint32_t rel = __ballot_sync(FULL, foot != 0u);
+    const uint32_t below = rel & ((1u << lane) - 1u);
+    const int prev = below ? 31 - __clz(below) : -1;
+    const uint32_t prev_end = __shfl_sync(FULL, (c == foot) ? a + c : 0xFFFFFFFFu, prev < 0 ? 0 : prev);
+    const bool head = c != 0u && (prev < 0 || prev_end != a);
     const uint32_t heads = __ballot_sync(FULL, head);
     const uint32_t above = lane == 31 ? 0u : heads & (0xFFFFFFFFu << (lane + 1));  // heads above this lane
     const uint32_t next = above ? (uint32_t)(__ffs(above) - 1) : 32u;
