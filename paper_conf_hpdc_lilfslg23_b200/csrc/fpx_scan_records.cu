@@ -177,21 +177,22 @@ struct Witness {
     mn64 = min(mn64, a3 - 1u);
     mx64 = max(mx64, a3);
   }
+  // packed halves: per-halfword DPX min / max (VIADDMNMX.U16x2, VIMNMX.U16x2)
   template <bool BF>
   __device__ __forceinline__ void half2(uint32_t x) {
     x &= 0x7FFF7FFFu;
-    const uint32_t l = x & 0xFFFFu, h = x >> 16;
     if (BF) {
-      mnb = min(mnb, min(l - 1u, h - 1u));
-      mxb = max(mxb, max(l, h));
+      mnb = __viaddmin_u16x2(x, 0xFFFFFFFFu, mnb);  // h - 1 per half (0 -> 0xFFFF)
+      mxb = __vimax3_u16x2(x, x, mxb);
     } else {
-      mn16 = min(mn16, min(l - 1u, h - 1u));
-      mx16 = max(mx16, max(l, h));
+      mn16 = __viaddmin_u16x2(x, 0xFFFFFFFFu, mn16);
+      mx16 = __vimax3_u16x2(x, x, mx16);
     }
   }
   __device__ __forceinline__ bool hit() const {
     return mn32 < 0x00FFFFFEu || mx32 >= 0xFF000000u || mn64 < 0x000FFFFFu || mx64 >= 0x7FF00000u ||
-           mn16 < 0x03FFu || mx16 > 0x7BFFu || mnb < 0x007Fu || mxb > 0x7F7Fu;
+           min(mn16 & 0xFFFFu, mn16 >> 16) < 0x03FFu || max(mx16 & 0xFFFFu, mx16 >> 16) > 0x7BFFu ||
+           min(mnb & 0xFFFFu, mnb >> 16) < 0x007Fu || max(mxb & 0xFFFFu, mxb >> 16) > 0x7F7Fu;
   }
 };
 

@@ -46,39 +46,42 @@ __device__ __forceinline__ uint32_t vec_cls(const uint4& q, uint32_t e) {
 // Cheap "anything exceptional in this vector" witness update.
 template <uint32_t FMT>
 __device__ __forceinline__ void vec_witness(const uint4& q, uint32_t& mn, uint32_t& mx) {
+  // Exact witnesses (see witness_hit): FP32 a2 = |x| << 1 (x + x: FMA pipe);
+  // FP64 a3 = |hi| | (lo != 0); packed halves per halfword.
   if (FMT == FPX_FP32) {
     const uint32_t w[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
-      const uint32_t a = w[k] & 0x7FFFFFFFu;
-      mn = min(mn, a - 1u);
-      mx = max(mx, a);
+      const uint32_t a2 = w[k] + w[k];
+      mn = min(mn, a2 - 2u);
+      mx = max(mx, a2);
     }
   } else if (FMT == FPX_FP64) {
     const uint32_t lo[2] = {q.x, q.z}, hi[2] = {q.y, q.w};
 #pragma unroll
     for (int k = 0; k < 2; ++k) {
-      const uint32_t a2 = ((hi[k] & 0x7FFFFFFFu) << 1) | min(lo[k], 1u);
-      mn = min(mn, a2 - 1u);
-      mx = max(mx, a2);
+      const uint32_t a3 = (hi[k] & 0x7FFFFFFFu) | min(lo[k], 1u);
+      mn = min(mn, a3 - 1u);
+      mx = max(mx, a3);
     }
   } else {
-    const uint32_t w[4] = {q.x, q.y, q.z, q.w};
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const uint32_t x = w[k] & 0x7FFF7FFFu;
-      const uint32_t l = x & 0xFFFFu, h = x >> 16;
-      mn = min(mn, min(l - 1u, h - 1u));
-      mx = max(mx, max(l, h));
-    }
+    // packed halves: per-halfword DPX min / max (VIADDMNMX.U16x2, VIMNMX3.U16x2)
+    const uint32_t a = q.x & 0x7FFF7FFFu, b = q.y & 0x7FFF7FFFu, c = q.z & 0x7FFF7FFFu, d = q.w & 0x7FFF7FFFu;
+    mn = __viaddmin_u16x2(a, 0xFFFFFFFFu, mn);  // h - 1 per half (0 -> 0xFFFF)
+    mn = __viaddmin_u16x2(b, 0xFFFFFFFFu, mn);
+    mn = __viaddmin_u16x2(c, 0xFFFFFFFFu, mn);
+    mn = __viaddmin_u16x2(d, 0xFFFFFFFFu, mn);
+    mx = __vimax3_u16x2(a, b, mx);
+    mx = __vimax3_u16x2(c, d, mx);
   }
 }
 template <uint32_t FMT>
 __device__ __forceinline__ bool witness_hit(uint32_t mn, uint32_t mx) {
-  if (FMT == FPX_FP32) return mn < 0x007FFFFFu || mx > 0x7F7FFFFFu;
-  if (FMT == FPX_FP64) return mn < 0x001FFFFFu || mx >= 0xFFE00000u;
-  if (FMT == FPX_FP16) return mn < 0x03FFu || mx > 0x7BFFu;
-  return mn < 0x007Fu || mx > 0x7F7Fu;
+  if (FMT == FPX_FP32) return mn < 0x00FFFFFEu || mx >= 0xFF000000u;  // subnormal | INF/NaN
+  if (FMT == FPX_FP64) return mn < 0x000FFFFFu || mx >= 0x7FF00000u;
+  const uint32_t lo = min(mn & 0xFFFFu, mn >> 16), hi = max(mx & 0xFFFFu, mx >> 16);
+  if (FMT == FPX_FP16) return lo < 0x03FFu || hi > 0x7BFFu;
+  return lo < 0x007Fu || hi > 0x7F7Fu;
 }
 
 constexpr int TU = 4;  // vectors per thread per batch
