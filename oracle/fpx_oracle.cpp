@@ -26,6 +26,13 @@
 // The loops follow the definition literally: record by record, lane by lane,
 // value by value, one map update per exceptional lane-value.  No blocking, no
 // warp aggregation, no hashing.
+//
+// Pins: tests/test_oracle_pins.py (exhaustive closed forms, numpy IEEE
+// predicates, the paper's worked cases, brute force through real IEEE ops,
+// planted-event aggregates).  Parity unpinned by the paper: the KILL kind
+// when several sources are exceptional (severity order NaN > INF > SUB,
+// reading R5) and per-half counting of packed FP16/BF16 values (R13) are
+// conventions of DESIGN.md §3, pinned only to that text.
 
 #include <cstdint>
 #include <cstring>
