@@ -100,3 +100,24 @@ def test_t4_summary_counts_distinct_sites():
     e["kind"] = [0, 0, 0, 2, 1]
     e["flow"] = [0, 1, 2, 0, 0]
     assert fpx.t4_summary(e) == {(0, 0): 2, (1, 2): 1, (0, 1): 1}
+
+
+def test_report_lines_and_t4():
+    from paper_conf_hpdc_lilfslg23_b200 import fpx, report
+
+    e = np.zeros(4, dtype=fpx.ENTRY_DTYPE)
+    e["site"] = [0x10002, 0x10002, 0x30001, 0x30001]
+    e["fmt"] = [0, 0, 1, 1]
+    e["kind"] = [0, 3, 1, 2]
+    e["flow"] = [0, 0, 2, 3]
+    e["count"] = [5, 1, 7, 2]
+    e["first_index"] = [10, 11, 12, 13]
+    names = {0x10002: ("ampere_sgemm_32x128_nn", "/unknown_path")}
+    det = report.detector_lines(e, names)
+    assert det[0].startswith("#GPU-FPX LOC-EXCEP INFO: in kernel [ampere_sgemm_32x128_nn], NaN found @ /unknown_path")
+    assert det[0].endswith("[FP32] count=5 first=10") and "DIV0 found" in det[1] and len(det) == 2
+    ana = report.analyzer_lines(e)
+    assert ana[0].startswith("#GPU-FPX-ANA PROPAGATION: INF") and "[FP64]" in ana[0]
+    assert ana[1].startswith("#GPU-FPX-ANA DISAPPEARANCE: SUB")
+    assert report.t4_table(e) == {(0, 0): 1, (0, 3): 1, (1, 1): 1, (1, 2): 1}
+    assert report.t4_lines(e)[1].split() == ["FP32", "1", "0", "0", "1"]

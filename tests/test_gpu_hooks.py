@@ -1,0 +1,33 @@
+"""the activation detector finds the first module whose output
+holds NaN / INF (the SRU uninitialised-tensor case, recast for
+model code), through fpx_scan_tensor forward hooks."""
+import pytest
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+
+def test_activation_scanner_finds_first_nan_module():
+    from paper_conf_hpdc_lilfslg23_b200.hooks import ActivationScanner
+    from paper_conf_hpdc_lilfslg23_b200 import fpx
+
+    torch.manual_seed(0)
+    model = torch.nn.Sequential(
+        torch.nn.Linear(64, 128), torch.nn.ReLU(), torch.nn.Linear(128, 128), torch.nn.Tanh(),
+        torch.nn.Linear(128, 10),
+    ).cuda()
+    x = torch.randn(32, 64, device="cuda")
+    sc = ActivationScanner(model)
+    model(x)
+    assert sc.first_exception() is None  # clean forward
+    with torch.no_grad():
+        model[2].weight[5, 7] = float("nan")  # poison the second Linear
+    model(x)
+    model(x)
+    call, name, element, kind = sc.first_exception()
+    assert (call, name, kind) == (2, "2", fpx.NAN)
+    assert element % 128 == 5  # output column 5 of the first row that reaches it
+    ents = sc.entries()
+    sites = {sc.names[int(e["site"])] for e in ents}
+    assert sites == {"2", "3", "4"}  # NaN propagates to every later layer
+    sc.remove()
