@@ -409,9 +409,9 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 // Ring configurations compiled in; FPX_RING (environment, tuning only) picks
 // one, default RING_DEFAULT.
 using Ring0 = RingCfg<16, 2, 48>;
-using Ring1 = RingCfg<8, 3, 64>;
-using Ring2 = RingCfg<12, 2, 64>;
-using Ring3 = RingCfg<16, 2, 32>;
+using Ring1 = RingCfg<20, 2, 36>;
+using Ring2 = RingCfg<24, 2, 28>;
+using Ring3 = RingCfg<18, 2, 42>;
 static_assert(ring_smem<Ring0>() <= 227 * 1024 && ring_smem<Ring1>() <= 227 * 1024 &&
                   ring_smem<Ring2>() <= 227 * 1024 && ring_smem<Ring3>() <= 227 * 1024,
               "ring exceeds shared memory");
@@ -591,11 +591,17 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
                                                                          d_arena, arena_planes, base_index, tv);
     return cudaGetLastError();
   }
-  static int ring = -1;
-  if (ring < 0) {
+  // Ring geometry: big stages pay off when records carry several planes (per
+  // tile fixed work is amortised over more bytes), more warps when they carry
+  // about one (C5-like FP32 traces).  Estimated from the arena density;
+  // FPX_RING (environment, tuning only) overrides.
+  static int forced = -2;
+  if (forced == -2) {
     const char* e = getenv("FPX_RING");
-    ring = e ? atoi(e) : 0;
+    forced = e ? atoi(e) : -1;
   }
+  int ring = forced;
+  if (ring < 0) ring = (arena_planes * 4 < n * 5) ? 1 : 0;  // < 1.25 planes per record -> 20-warp ring
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   switch (ring) {
     case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
