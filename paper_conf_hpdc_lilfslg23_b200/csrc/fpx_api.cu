@@ -178,13 +178,16 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   const uint64_t cap = o.newlog_capacity ? std::min<uint64_t>(o.newlog_capacity, h->slots) : h->slots;
   Slot* slots = nullptr;
   unsigned long long* log = nullptr;
+  unsigned int* log_slot = nullptr;
   Ctl* ctl = nullptr;
   if (cudaMalloc(&slots, sizeof(Slot) * h->slots) != cudaSuccess ||
       cudaMalloc(&log, sizeof(unsigned long long) * cap) != cudaSuccess ||
+      cudaMalloc(&log_slot, sizeof(unsigned int) * cap) != cudaSuccess ||
       cudaMalloc(&ctl, sizeof(Ctl)) != cudaSuccess || cudaMallocHost(&h->h_ctl, sizeof(Ctl)) != cudaSuccess) {
     cudaGetLastError();
     if (slots) cudaFree(slots);
     if (log) cudaFree(log);
+    if (log_slot) cudaFree(log_slot);
     if (ctl) cudaFree(ctl);
     delete h;
     return FPX_ERR_NOMEM;
@@ -192,6 +195,7 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   h->tv.slots = slots;
   h->tv.mask = h->slots - 1;
   h->tv.newlog = log;
+  h->tv.newlog_slot = log_slot;
   h->tv.newlog_cap = cap;
   h->tv.ctl = ctl;
   CK(launch_table_reset(h->tv, h->slots, nullptr));
@@ -359,7 +363,7 @@ fpx_status fpx_table_reset(fpx_handle h, void* stream) {
   if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   if (h->last_stream != s) CK(cudaStreamSynchronize(h->last_stream));
-  CK(launch_table_reset(h->tv, h->slots, s));
+  CK(launch_table_reset_touched(h->tv, h->slots, s));
   h->newlog_cursor = 0;
   h->last_stream = s;
   return FPX_OK;
@@ -385,6 +389,7 @@ fpx_status fpx_close(fpx_handle h) {
     cudaDeviceSynchronize();
     cudaFree(h->tv.slots);
     cudaFree(h->tv.newlog);
+    cudaFree(h->tv.newlog_slot);
     cudaFree(h->tv.ctl);
     cudaFreeHost(h->h_ctl);
     for (void* p : {(void*)h->d_keys, (void*)h->d_counts, (void*)h->d_first, (void*)h->d_keys2, (void*)h->d_idx,

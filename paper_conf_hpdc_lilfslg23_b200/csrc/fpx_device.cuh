@@ -115,8 +115,12 @@ static __device__ __noinline__ void table_add(const TableView tv, unsigned long 
       if (k == FPX_KEY_EMPTY) {
         // this thread inserted the key: log it once (the "new combination")
         unsigned long long pos = atomicAdd(&tv.ctl->newlog_tail, 1ull);
-        if (pos < tv.newlog_cap) tv.newlog[pos] = key;
-        else atomicAdd(&tv.ctl->newlog_overflow, 1ull);
+        if (pos < tv.newlog_cap) {
+          tv.newlog[pos] = key;
+          tv.newlog_slot[pos] = (unsigned int)i;
+        } else {
+          atomicAdd(&tv.ctl->newlog_overflow, 1ull);
+        }
         k = key;
       }
     }

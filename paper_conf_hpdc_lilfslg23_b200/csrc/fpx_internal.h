@@ -37,6 +37,7 @@ struct TableView {
   Slot* slots;
   unsigned long long mask;       // slots - 1
   unsigned long long* newlog;
+  unsigned int* newlog_slot;     // slot index of each logged key (for the touched-slot reset)
   unsigned long long newlog_cap;
   Ctl* ctl;
 };
@@ -49,6 +50,10 @@ cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint
 cudaError_t launch_scan_tensor(const void* d_ptr, uint64_t n_elems, uint32_t fmt, uint32_t site,
                                uint64_t base_index, const TableView& tv, int num_sms, cudaStream_t s);
 cudaError_t launch_table_reset(const TableView& tv, uint64_t slots, cudaStream_t s);
+// Clear only the slots recorded in the new-key log (every occupied slot is
+// there unless the log overflowed, in which case the whole table is cleared),
+// then the counters.  O(entries) instead of O(slots); stream-ordered, no sync.
+cudaError_t launch_table_reset_touched(const TableView& tv, uint64_t slots, cudaStream_t s);
 // Compact non-empty slots into (keys, counts, firsts); *d_n receives the count.
 cudaError_t launch_table_compact(const TableView& tv, uint64_t slots, uint64_t* d_keys,
                                  uint64_t* d_counts, uint64_t* d_first, unsigned long long* d_n,

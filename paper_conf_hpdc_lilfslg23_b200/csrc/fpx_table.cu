@@ -33,6 +33,34 @@ __global__ void k_reset(Slot* slots, uint64_t n, Ctl* ctl) {
   }
 }
 
+__device__ __forceinline__ void clear_slot(Slot* slots, uint64_t i) {
+  Slot s;
+  s.key = FPX_KEY_EMPTY;
+  s.count = 0;
+  s.first = ~0ull;
+  s.pad = 0;
+  slots[i] = s;
+}
+
+// every occupied slot was logged at insert (unless the log overflowed)
+__global__ void k_reset_touched(const TableView tv, uint64_t slots) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t t0 = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  const unsigned long long tail = tv.ctl->newlog_tail;
+  if (tv.ctl->newlog_overflow != 0 || tail > tv.newlog_cap) {
+    for (uint64_t i = t0; i < slots; i += stride) clear_slot(tv.slots, i);
+  } else {
+    for (uint64_t i = t0; i < tail; i += stride) clear_slot(tv.slots, tv.newlog_slot[i]);
+  }
+}
+
+__global__ void k_reset_ctl(Ctl* ctl) {
+  ctl->bad_records = 0;
+  ctl->dropped_events = 0;
+  ctl->newlog_tail = 0;
+  ctl->newlog_overflow = 0;
+}
+
 __global__ void k_compact(const Slot* slots, uint64_t n, uint64_t* keys, uint64_t* counts, uint64_t* firsts,
                           unsigned long long* d_n) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
@@ -108,6 +136,14 @@ unsigned grid_for(uint64_t n) {
 
 cudaError_t launch_table_reset(const TableView& tv, uint64_t slots, cudaStream_t s) {
   k_reset<<<grid_for(slots), 256, 0, s>>>(tv.slots, slots, tv.ctl);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_table_reset_touched(const TableView& tv, uint64_t slots, cudaStream_t s) {
+  k_reset_touched<<<148 * 4, 256, 0, s>>>(tv, slots);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  k_reset_ctl<<<1, 1, 0, s>>>(tv.ctl);
   return cudaGetLastError();
 }
 

@@ -336,3 +336,22 @@ def test_generator_device_matches_host(recipe):
     fpxgen.apply_host(w, hdr, arena)
     fpxgen.apply_device(w, d_hdr, d_arena)
     assert np.array_equal(d_arena[: planes * 32].cpu().numpy().view(np.uint32), arena.reshape(-1))
+
+
+@pytest.mark.parametrize("newlog_capacity", [0, 8])  # 8 < keys: the log overflows -> full clear
+def test_reset_clears_every_key(fpx, newlog_capacity):
+    p = fpxgen.Params(seed=3, n_records=30_000, n_sites=500, recipe=fpxgen.RECIPE_MIX)
+    hdr, arena = fpxgen.generate_host(p)
+    _, w = fpxgen.plan_injections(p, 300)
+    fpxgen.apply_host(w, hdr, arena)
+    d_hdr, d_arena = to_dev(hdr, arena)
+    ref = oracle_scan(hdr, arena).entries()
+    with fpx.Handle(0, table_log2_slots=12, newlog_capacity=newlog_capacity) as h:
+        for rep in range(3):
+            h.scan_records(d_hdr, d_arena)
+            got = h.fetch()
+            assert_same(got, ref)
+            st = h.stats()
+            assert st.newlog_overflow == (0 if newlog_capacity == 0 else len(ref) - newlog_capacity)
+            h.reset()
+            assert len(h.fetch()) == 0 and h.stats().table_entries == 0
