@@ -531,7 +531,10 @@ def main():
             "peak_source": peak_src,
         },
         "clocks": clocks,
-        "gpu_launches": K * (2 + (3 + 2 if world > 1 else 0)),
+        # per step: table reset (2 kernels) + scan (1); merge (N > 1): compact, iota,
+        # radix sort, gather, sort, select-init, select, lookup (counted with ncu,
+        # tools/count_merge_launches.py); NCCL's own kernels are not ours
+        "gpu_launches": K * (3 + (8 if world > 1 else 0)),
         "cpu_baseline": cpu,
         "e2e": e2e,
     }

@@ -184,9 +184,7 @@ class Handle:
         dev = torch.device("cuda", self.device)
         n = ctypes.c_uint64(0)
         if capacity is None:
-            st = check(lib.fpx_table_fetch_device(self._h, None, None, None, 0, ctypes.byref(n), _stream_ptr(stream)),
-                       "fpx_table_fetch_device", allow=(ERR_TRUNCATED, ERR_BAD_RECORD, ERR_TABLE_FULL))
-            capacity = n.value
+            capacity = int(self.stats().table_entries)  # exact upper bound, no extra fetch pass
         k = torch.empty(max(capacity, 1), dtype=torch.int64, device=dev)
         c = torch.empty_like(k)
         f = torch.empty_like(k)
