@@ -149,6 +149,32 @@ __device__ __noinline__ void exact_tile(const RecDesc* __restrict__ recs, const 
   }
 }
 
+// Same as exact_tile, reading the tile's k headers from global memory (the
+// record-scan ring keeps no header copy in shared memory).
+template <int MODE>
+__device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
+                                            const uint32_t* __restrict__ lane_base, int lane, uint64_t gidx0,
+                                            const TableView tv) {
+  uint4 h = make_uint4(0u, 0u, 0u, 0u);
+  if ((uint32_t)lane < k) h = hdr_tile[lane];
+  const bool ok = (uint32_t)lane < k && record_valid<MODE>(h, arena_planes);
+  const uint32_t mask = ok ? h.y : 0u;
+  for (uint32_t j = 0; j < k; ++j) {
+    const RecDesc d{__shfl_sync(FULL, h.w, j), __shfl_sync(FULL, mask, j), __shfl_sync(FULL, h.z, j),
+                    __shfl_sync(FULL, h.x, j)};
+    if (d.mask == 0u) continue;  // warp-uniform
+    if (MODE == FPX_MODE_DEST && is_compare(op_of(d.meta))) continue;
+    uint32_t codes, evm;
+    const uint32_t cm = eval_record<MODE>(d, lane_base, lane, codes, evm);
+    warp_flush(tv, cm, d.site, fmt_of(d.meta), gidx0 + j, [&](int c) {
+      uint32_t nn = 0;
+#pragma unroll
+      for (int v = 0; v < 8; ++v) nn += (((evm >> v) & 1u) && (((codes >> (4 * v)) & 15u) == (uint32_t)c)) ? 1u : 0u;
+      return nn;
+    });
+  }
+}
+
 // Plane items of one record for the fast path, by list:
 //   0: FP32 words, 1: FP64 (lo, hi) pairs, 2: FP16x2 words, 3: BF16x2 words.
 template <int MODE>

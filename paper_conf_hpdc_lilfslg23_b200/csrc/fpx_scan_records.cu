@@ -115,7 +115,6 @@ template <class C>
 struct WarpSmem {
   uint32_t planes[C::STAGES][C::PLANES * 32];  // 128 B per plane
   uint2 items[C::STAGES][C::PLANES];           // {plane slot, active mask}
-  RecDesc recs[C::STAGES][TILE];
   StageMeta meta[C::STAGES];
   uint64_t bar[C::STAGES];
 };
@@ -326,7 +325,6 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     // order those generic reads before the async-proxy writes below
     __syncwarp();
     fence_proxy_async_smem();
-    sm.recs[s][lane] = in_tile ? RecDesc{h.w, mask, h.z, h.x} : RecDesc{0u, 0u, 0u, 0u};
     // list l = 2 * fmt + partial; lists of lower formats come first
     const uint32_t tot_f = tf + tp;  // packed per-format item totals (<= 128 each)
     if (in_tile && ni != 0u) {
@@ -402,16 +400,17 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       consume_list<FPX_BF16, false>(w, seg[6], seg[7], ia, pa, g, q);
       consume_list<FPX_BF16, true>(w, seg[7], seg[8], ia, pa, g, q);
     }
-    if (__any_sync(FULL, w.hit()) || m.force) exact_tile<MODE>(sm.recs[s], lane_base, lane, m.gidx0, tv);
+    if (__any_sync(FULL, w.hit()) || m.force)
+      exact_tile_hdr<MODE>(hdr + (m.gidx0 - base_index), m.k, arena_planes, lane_base, lane, m.gidx0, tv);
   }
 }
 
 // Ring configurations compiled in; FPX_RING (environment, tuning only) picks
 // one, default RING_DEFAULT.
-using Ring0 = RingCfg<16, 2, 48>;
-using Ring1 = RingCfg<20, 2, 36>;
-using Ring2 = RingCfg<24, 2, 28>;
-using Ring3 = RingCfg<18, 2, 42>;
+using Ring0 = RingCfg<16, 2, 50>;
+using Ring1 = RingCfg<20, 2, 40>;
+using Ring2 = RingCfg<16, 3, 32>;
+using Ring3 = RingCfg<18, 2, 44>;
 static_assert(ring_smem<Ring0>() <= 227 * 1024 && ring_smem<Ring1>() <= 227 * 1024 &&
                   ring_smem<Ring2>() <= 227 * 1024 && ring_smem<Ring3>() <= 227 * 1024,
               "ring exceeds shared memory");
