@@ -112,7 +112,7 @@ struct StageMeta {
 };
 
 template <class C>
-struct WarpSmem {
+struct alignas(128) WarpSmem {  // 128-B multiple: every warp's planes stay 16-B (TMA / LDS.128) aligned
   uint32_t planes[C::STAGES][C::PLANES * 32];  // 128 B per plane
   uint2 items[C::STAGES][C::PLANES];           // {plane slot, active mask}
   StageMeta meta[C::STAGES];
@@ -407,11 +407,11 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 
 // Ring configurations compiled in; FPX_RING (environment, tuning only) picks
 // one, default RING_DEFAULT.
-using Ring0 = RingCfg<16, 2, 50>;
+using Ring0 = RingCfg<16, 2, 52>;
 using Ring1 = RingCfg<20, 2, 40>;
 using Ring2 = RingCfg<16, 3, 32>;
-using Ring3 = RingCfg<18, 2, 44>;
-static_assert(ring_smem<Ring0>() <= 227 * 1024 && ring_smem<Ring1>() <= 227 * 1024 &&
+using Ring3 = RingCfg<18, 2, 46>;
+static_assert(sizeof(WarpSmem<Ring2>) % 128 == 0 && ring_smem<Ring0>() <= 227 * 1024 && ring_smem<Ring1>() <= 227 * 1024 &&
                   ring_smem<Ring2>() <= 227 * 1024 && ring_smem<Ring3>() <= 227 * 1024,
               "ring exceeds shared memory");
 
