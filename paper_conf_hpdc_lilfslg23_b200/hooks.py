@@ -18,10 +18,31 @@ from . import fpx
 SEQ_SHIFT = 36  # element indices below 2^36 per scanned output
 
 
+class SelectivePolicy:
+    """Alg3, selective instrumentation, at the API level: scan a
+    kernel / module only if it is in the white-list (when one is given) and
+    only on one in every k of its invocations (freq-redn-factor; k = 0 or 1:
+    every invocation).  ``num[name]`` counts invocations as in Alg3 line 14."""
+
+    def __init__(self, white_list=None, k: int = 0):
+        self.white = set(white_list) if white_list else None
+        self.k = k
+        self.num = {}
+
+    def should_scan(self, name: str) -> bool:
+        instr = self.white is None or name in self.white      # Alg3 lines 2-9
+        n = self.num.get(name, 0)
+        if self.k not in (0, 1) and n % self.k != 0:          # Alg3 lines 10-13
+            instr = False
+        self.num[name] = n + 1                                # Alg3 line 14
+        return instr
+
+
 class ActivationScanner:
     def __init__(self, model: torch.nn.Module, handle: "fpx.Handle | None" = None, leaf_only: bool = True,
-                 device: int | None = None):
+                 device: int | None = None, policy: SelectivePolicy | None = None):
         self.model = model
+        self.policy = policy
         dev = torch.cuda.current_device() if device is None else device
         self.handle = handle if handle is not None else fpx.Handle(dev)
         self._own = handle is None
@@ -42,7 +63,8 @@ class ActivationScanner:
 
     def _make_hook(self, site: int):
         def hook(module, args, out):
-            self._scan(out, site)
+            if self.policy is None or self.policy.should_scan(self.names[site]):
+                self._scan(out, site)
 
         return hook
 

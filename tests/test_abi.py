@@ -121,3 +121,21 @@ def test_report_lines_and_t4():
     assert ana[1].startswith("#GPU-FPX-ANA DISAPPEARANCE: SUB")
     assert report.t4_table(e) == {(0, 0): 1, (0, 3): 1, (1, 1): 1, (1, 2): 1}
     assert report.t4_lines(e)[1].split() == ["FP32", "1", "0", "0", "1"]
+
+
+def test_selective_policy_is_alg3():
+    import torch  # noqa: F401  (hooks imports torch)
+    from paper_conf_hpdc_lilfslg23_b200.hooks import SelectivePolicy
+
+    # no white-list, k = 0: every invocation (Alg3 lines 7-8)
+    p = SelectivePolicy()
+    assert all(p.should_scan("a") for _ in range(5))
+    # white-list only (lines 3-6)
+    p = SelectivePolicy(white_list={"a"})
+    assert [p.should_scan(x) for x in "abab"] == [True, False, True, False]
+    # 1 in k invocations per kernel, counted per name (lines 10-14)
+    p = SelectivePolicy(k=3)
+    assert [p.should_scan("a") for _ in range(7)] == [True, False, False, True, False, False, True]
+    assert p.should_scan("b") and p.num == {"a": 7, "b": 1}
+    p = SelectivePolicy(white_list={"a"}, k=2)
+    assert [p.should_scan(x) for x in "aabba"] == [True, False, False, False, True]

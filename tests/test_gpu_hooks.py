@@ -31,3 +31,20 @@ def test_activation_scanner_finds_first_nan_module():
     sites = {sc.names[int(e["site"])] for e in ents}
     assert sites == {"2", "3", "4"}  # NaN propagates to every later layer
     sc.remove()
+
+
+def test_activation_scanner_with_selective_policy():
+    from paper_conf_hpdc_lilfslg23_b200.hooks import ActivationScanner, SelectivePolicy
+
+    model = torch.nn.Sequential(torch.nn.Linear(16, 16), torch.nn.Linear(16, 16)).cuda()
+    with torch.no_grad():
+        model[0].weight[0, 0] = float("inf")
+    x = torch.ones(4, 16, device="cuda")
+    sc = ActivationScanner(model, policy=SelectivePolicy(white_list={"1"}, k=2))
+    for _ in range(4):
+        model(x)
+    ents = sc.entries()
+    # only module "1" is scanned, on forward calls 1 and 3 (1 in 2)
+    assert {sc.names[int(e["site"])] for e in ents} == {"1"}
+    assert len(sc.seq) == 2 and [c for c, _ in sc.seq] == [1, 3]
+    sc.remove()
