@@ -72,8 +72,21 @@ enum { FPX_NAN = 0, FPX_INF = 1, FPX_SUB = 2, FPX_DIV0 = 3 };
 enum { FPX_FLOW_NONE = 0, FPX_GEN = 1, FPX_PROP = 2, FPX_KILL = 3 };
 
 /* Scan modes: the detector (dest-only, §3.1) and the analyzer (flow, §3.2);
- * the two-phase workflow of Fig 2 / P:167, 230. */
-enum { FPX_MODE_DEST = 0, FPX_MODE_FLOW = 1 };
+ * the two-phase workflow of Fig 2 / P:167, 230.  FPX_MODE_FLOW_DETAIL is the
+ * analyzer plus Table 2's separate "Comparison" state and per-source
+ * attribution (fn4 P:99 "INF flowed from R3 to R1"): entries
+ * also carry `detail` (below). */
+enum { FPX_MODE_DEST = 0, FPX_MODE_FLOW = 1, FPX_MODE_FLOW_DETAIL = 2 };
+
+/* detail byte of an entry (0 outside FPX_MODE_FLOW_DETAIL):
+ *   bits [1:0]  1 + index of the source operand that set the source class S
+ *               (the lowest-index source with the most severe class), 0 if no
+ *               source was exceptional;
+ *   bit 2       FPX_DETAIL_CMP: the instruction is a control-flow opcode
+ *               (Table 1's right column: FSEL, FSET, FSETP, FMNMX, DSETP) and a
+ *               source was exceptional — Table 2's "Comparison" state. */
+#define FPX_DETAIL_SRC(d) ((uint32_t)(d) & 3u)
+#define FPX_DETAIL_CMP 4u
 
 /* Opcode classes (Table 1; Alg1 dispatch; SASS opcode -> opcode_id
  * map of P:332).  HADD2..HMMA are the FP16/BF16 "future" formats;
@@ -144,10 +157,12 @@ typedef struct {
 /* ------------------------------------------------------------------------ */
 /* Table key and entries                                                     */
 /* ------------------------------------------------------------------------ */
-/* key = site << 32 | fmt << 4 | flow << 2 | kind.  Ascending key order =
- * (site, fmt, flow, kind) order; fetch always returns entries in this order. */
+/* key = site << 32 | detail << 6 | fmt << 4 | flow << 2 | kind.  Ascending
+ * key order = (site, detail, fmt, flow, kind) order; fetch always returns
+ * entries in this order (detail is 0 except in FPX_MODE_FLOW_DETAIL). */
 #define FPX_KEY(site, fmt, flow, kind) \
   (((uint64_t)(site) << 32) | ((uint64_t)(fmt) << 4) | ((uint64_t)(flow) << 2) | (uint64_t)(kind))
+#define FPX_KEY_DETAIL(site, detail, fmt, flow, kind) (FPX_KEY(site, fmt, flow, kind) | ((uint64_t)(detail) << 6))
 #define FPX_KEY_EMPTY 0xFFFFFFFFFFFFFFFFull
 
 typedef struct {
@@ -155,7 +170,7 @@ typedef struct {
   uint8_t kind;          /* FPX_NAN..FPX_DIV0 */
   uint8_t flow;          /* FPX_FLOW_NONE..FPX_KILL */
   uint8_t fmt;           /* FPX_FP32..FPX_BF16 */
-  uint8_t _pad;
+  uint8_t detail;        /* FPX_MODE_FLOW_DETAIL attribution, else 0 */
   uint64_t count;        /* number of lane-values with this key */
   uint64_t first_index;  /* min base_index + record (or element) index */
 } fpx_entry;             /* 24 bytes */
@@ -195,12 +210,13 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out);
  *   d_arena    device pointer to arena_planes planes of 128 B (16-B aligned)
  *   base_index global index of d_hdr[0]; record r reports first_index
  *              base_index + r (lets a stream be scanned in batches / shards)
- *   mode       FPX_MODE_DEST (detector) or FPX_MODE_FLOW (analyzer)
+ *   mode       FPX_MODE_DEST (detector), FPX_MODE_FLOW (analyzer) or
+ *              FPX_MODE_FLOW_DETAIL (analyzer + Comparison state + source)
  * Every lane-value of every active lane is classified; per warp the events
  * are reduced before any atomic; the table gets count += lane-values,
  * first = min(first, base_index + r).  Records that fail validation (reserved
- * bits, enum ranges, planes outside the arena, invalid site, and in FLOW mode
- * records other than scalar FP32/FP64) are counted and skipped.
+ * bits, enum ranges, planes outside the arena, invalid site, and in the FLOW
+ * modes records other than scalar FP32/FP64) are counted and skipped.
  * n_records == 0 is a no-op.  Buffers must stay valid until the stream passes
  * the scan.  Errors: FPX_ERR_INVALID, FPX_ERR_CUDA. */
 fpx_status fpx_scan_records(fpx_handle h, const fpx_rec_hdr* d_hdr, uint64_t n_records,

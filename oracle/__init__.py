@@ -24,7 +24,7 @@ ENTRY_DTYPE = np.dtype(
         ("kind", "u1"),
         ("flow", "u1"),
         ("fmt", "u1"),
-        ("_pad", "u1"),
+        ("detail", "u1"),
         ("count", "<u8"),
         ("first_index", "<u8"),
     ]

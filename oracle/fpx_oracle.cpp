@@ -48,10 +48,10 @@ constexpr uint32_t K_NAN = 0, K_INF = 1, K_SUB = 2, K_DIV0 = 3;
 // Table 2 states: none (detector), Appearance, Propagation,
 // Disappearance.
 constexpr uint32_t F_NONE = 0, F_GEN = 1, F_PROP = 2, F_KILL = 3;
-constexpr uint32_t MODE_DEST = 0, MODE_FLOW = 1;
+constexpr uint32_t MODE_DEST = 0, MODE_FLOW = 1, MODE_FLOW_DETAIL = 2;
 // Opcode classes (Table 1 P:101-110 plus the packed / synthetic ones).
-constexpr uint32_t OP_MUFU_RCP = 4, OP_MUFU_RCP64H = 5, OP_FSET = 11, OP_FSETP = 12,
-                   OP_DSETP = 14, OP_DIV = 19, OP_COUNT = 20;
+constexpr uint32_t OP_MUFU_RCP = 4, OP_MUFU_RCP64H = 5, OP_FSEL = 10, OP_FSET = 11, OP_FSETP = 12,
+                   OP_FMNMX = 13, OP_DSETP = 14, OP_DIV = 19, OP_COUNT = 20;
 
 // Value classes of §2.1.
 enum Cls { CLEAN = 0, C_NAN = 1, C_INF = 2, C_SUB = 3 };
@@ -63,7 +63,7 @@ static_assert(sizeof(Hdr) == 16, "header is 16 bytes");
 
 struct Entry {  // fetched entry, 24 bytes
   uint32_t site;
-  uint8_t kind, flow, fmt, pad;
+  uint8_t kind, flow, fmt, detail;
   uint64_t count, first_index;
 };
 static_assert(sizeof(Entry) == 24, "entry is 24 bytes");
@@ -155,8 +155,13 @@ uint32_t dest_kind(uint32_t opclass, uint32_t fmt, uint64_t d,
   return c == CLEAN ? NO_KIND : kind_of(c);
 }
 
-uint64_t make_key(uint32_t site, uint32_t fmt, uint32_t flow, uint32_t kind) {
-  return ((uint64_t)site << 32) | ((uint64_t)fmt << 4) | ((uint64_t)flow << 2) | kind;
+uint64_t make_key(uint32_t site, uint32_t fmt, uint32_t flow, uint32_t kind, uint32_t detail = 0) {
+  return ((uint64_t)site << 32) | ((uint64_t)detail << 6) | ((uint64_t)fmt << 4) | ((uint64_t)flow << 2) | kind;
+}
+
+// Control-flow opcodes of Table 1's right column.
+bool is_control_flow(uint32_t op) {
+  return op == OP_FSEL || op == OP_FSET || op == OP_FSETP || op == OP_FMNMX || op == OP_DSETP;
 }
 
 }  // namespace
@@ -170,8 +175,8 @@ struct orc_table {
 namespace {
 
 void record_event(orc_table* t, uint32_t site, uint32_t fmt, uint32_t flow, uint32_t kind,
-                  uint64_t g) {
-  Val& e = t->gt[make_key(site, fmt, flow, kind)];
+                  uint64_t g, uint32_t detail = 0) {
+  Val& e = t->gt[make_key(site, fmt, flow, kind, detail)];
   e.count += 1;
   if (g < e.first) e.first = g;
 }
@@ -187,7 +192,7 @@ bool record_valid(const Hdr& h, uint64_t arena_planes, uint32_t mode) {
   if (fmt == FMT_FP64 && (dwords % 2) != 0) return false;
   uint64_t planes = dwords + (uint64_t)nsrc * source_words(fmt);
   if ((uint64_t)h.val_off + planes > arena_planes) return false;
-  if (mode == MODE_FLOW) {
+  if (mode != MODE_DEST) {
     // FLOW is defined for scalar FP32 / FP64 records only (R13).
     if (fmt != FMT_FP32 && fmt != FMT_FP64) return false;
     if (dwords != 0 && dwords != source_words(fmt)) return false;
@@ -259,21 +264,29 @@ void orc_scan_records(orc_table* t, const void* hdr_v, uint64_t n, const uint32_
         }
       } else {
         // Analyzer: S = most severe class among the PRE-execution source
-        // values of this lane (R5).  Scalar records only (R13).
+        // values of this lane (R5); src = the lowest-index source
+        // holding that class (R21).  Scalar records only (R13).
         t->lane_values += n_dest + nsrc;
         Cls S = CLEAN;
+        uint32_t src = 0;
         for (uint32_t k = 0; k < nsrc; ++k) {
           s[k] = value_bits(fmt, sv[k], 0);
           Cls c = classify(fmt, s[k]);
-          if (severity(c) > severity(S)) S = c;
+          if (severity(c) > severity(S)) { S = c; src = k; }
         }
         uint32_t D = NO_KIND;
         if (n_dest == 1) D = dest_kind(opclass, fmt, value_bits(fmt, dw, 0), s, nsrc);
+        // FLOW_DETAIL: which source, and Table 2's Comparison state (R22)
+        uint32_t detail = 0;
+        if (mode == MODE_FLOW_DETAIL && S != CLEAN) {
+          detail = src + 1;
+          if (is_control_flow(opclass)) detail |= 4;
+        }
         // Table 2: Appearance (dest EV, no source EV), Propagation (dest EV,
         // source EV), Disappearance (no dest exception, source EV).
-        if (D != NO_KIND && S == CLEAN) record_event(t, h.site, fmt, F_GEN, D, g);
-        else if (D != NO_KIND && S != CLEAN) record_event(t, h.site, fmt, F_PROP, D, g);
-        else if (D == NO_KIND && S != CLEAN) record_event(t, h.site, fmt, F_KILL, kind_of(S), g);
+        if (D != NO_KIND && S == CLEAN) record_event(t, h.site, fmt, F_GEN, D, g, detail);
+        else if (D != NO_KIND && S != CLEAN) record_event(t, h.site, fmt, F_PROP, D, g, detail);
+        else if (D == NO_KIND && S != CLEAN) record_event(t, h.site, fmt, F_KILL, kind_of(S), g, detail);
       }
     }
   }
@@ -310,6 +323,7 @@ uint64_t orc_fetch(const orc_table* t, void* out_v, uint64_t cap) {
     e.fmt = (uint8_t)((kv.first >> 4) & 3);
     e.flow = (uint8_t)((kv.first >> 2) & 3);
     e.kind = (uint8_t)(kv.first & 3);
+    e.detail = (uint8_t)((kv.first >> 6) & 7);
     e.count = kv.second.count;
     e.first_index = kv.second.first;
     out[i++] = e;

@@ -25,13 +25,14 @@ OK, ERR_INVALID, ERR_CUDA, ERR_NOMEM, ERR_TABLE_FULL, ERR_BAD_RECORD, ERR_TRUNCA
 FP32, FP64, FP16, BF16 = 0, 1, 2, 3
 NAN, INF, SUB, DIV0 = 0, 1, 2, 3
 FLOW_NONE, GEN, PROP, KILL = 0, 1, 2, 3
-MODE_DEST, MODE_FLOW = 0, 1
+MODE_DEST, MODE_FLOW, MODE_FLOW_DETAIL = 0, 1, 2
+DETAIL_CMP = 4
 FETCH_ALL, FETCH_NEW = 0, 1
 OPT_SCAN_LDG = 1
 KEY_EMPTY = 0xFFFFFFFFFFFFFFFF
 
 ENTRY_DTYPE = np.dtype(
-    [("site", "<u4"), ("kind", "u1"), ("flow", "u1"), ("fmt", "u1"), ("_pad", "u1"), ("count", "<u8"),
+    [("site", "<u4"), ("kind", "u1"), ("flow", "u1"), ("fmt", "u1"), ("detail", "u1"), ("count", "<u8"),
      ("first_index", "<u8")]
 )
 HDR_DTYPE = np.dtype([("site", "<u4"), ("active_mask", "<u4"), ("meta", "<u4"), ("val_off", "<u4")])

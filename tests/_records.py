@@ -14,12 +14,12 @@ import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 HDR_DTYPE = np.dtype([("site", "<u4"), ("active_mask", "<u4"), ("meta", "<u4"), ("val_off", "<u4")])
-ENTRY_FIELDS = ("site", "kind", "flow", "fmt", "count", "first_index")
+ENTRY_FIELDS = ("site", "kind", "flow", "fmt", "detail", "count", "first_index")
 
 FP32, FP64, FP16, BF16 = 0, 1, 2, 3
 NAN, INF, SUB, DIV0 = 0, 1, 2, 3
 NONE, GEN, PROP, KILL = 0, 1, 2, 3
-DEST, FLOW = 0, 1
+DEST, FLOW, FLOW_DETAIL = 0, 1, 2
 OP_FADD, OP_FMUL, OP_FFMA, OP_RCP, OP_RCP64H, OP_MUFU = 1, 2, 3, 4, 5, 6
 OP_DADD, OP_DMUL, OP_DFMA, OP_FSEL, OP_FSET, OP_FSETP, OP_FMNMX, OP_DSETP = 7, 8, 9, 10, 11, 12, 13, 14
 OP_HADD2, OP_HFMA2, OP_HMUL2, OP_HMMA, OP_DIV = 15, 16, 17, 18, 19

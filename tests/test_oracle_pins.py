@@ -17,7 +17,7 @@ import pytest
 import fpxgen
 import oracle
 from _records import (
-    BF16, DEST, DIV0, FLOW, FP16, FP32, FP64, GEN, INF, KILL, NAN, NONE, OP_DIV, OP_FADD, OP_FFMA,
+    BF16, DEST, DIV0, FLOW, FLOW_DETAIL, FP16, FP32, FP64, GEN, INF, KILL, NAN, NONE, OP_DIV, OP_FADD, OP_FFMA,
     OP_FMNMX, OP_FMUL, OP_FSEL, OP_FSETP, OP_RCP, OP_RCP64H, PROP, SUB, Trace, expected_from_injections,
     load_worked_cases, np_class, table_dict, words_of,
 )
@@ -104,7 +104,7 @@ def _run_case(case, mode):
 
 @pytest.mark.parametrize("case", load_worked_cases(), ids=lambda c: c["name"])
 def test_worked_case(case):
-    for mode, key in ((DEST, "expect_dest"), (FLOW, "expect_flow")):
+    for mode, key in ((DEST, "expect_dest"), (FLOW, "expect_flow"), (FLOW_DETAIL, "expect_flow")):
         ents, r = _run_case(case, mode)
         exp = case[key]
         if exp is None:
@@ -115,6 +115,7 @@ def test_worked_case(case):
             assert (int(e["kind"]), int(e["flow"])) == tuple(exp), (mode, e)
             assert int(e["site"]) == 77 and int(e["fmt"]) == case["fmt"]
             assert int(e["count"]) == 5 and int(e["first_index"]) == 1000 + r
+            assert int(e["detail"]) == (case["expect_detail"] if mode == FLOW_DETAIL else 0), (mode, e)
 
 
 # --------------------------------------------------------------------------
@@ -159,7 +160,15 @@ def _ieee_expect(fmt, op, dest, srcs):
         fl = (S, KILL)
     else:
         fl = None
-    return (None if D is None else (D, NONE)), fl
+    # FLOW_DETAIL: 1 + lowest index of a source with the most severe class,
+    # | 4 for Table 1's control-flow opcodes (Table 2 "Comparison")
+    det = 0
+    if S is not None:
+        classes = [cls(s) for s in srcs]
+        det = 1 + next(i for i, c in enumerate(classes) if sev[c] == max(sev[x] for x in classes))
+        if op in (OP_FSEL, OP_FSETP, OP_FMNMX):
+            det |= 4
+    return (None if D is None else (D, NONE)), fl, det
 
 
 def _brute_records(fmt):
@@ -197,8 +206,8 @@ def test_bruteforce_ieee_ops(fmt):
         tr.add_value_record(9, opmap[op], fmt, 0xFFFFFFFF, None if dest is None else _bits(fmt, dest),
                             [_bits(fmt, s) for s in srcs])
         hdr, arena = tr.arrays()
-        exp_d, exp_f = _ieee_expect(fmt, op, dest, srcs)
-        for mode, exp in ((DEST, exp_d), (FLOW, exp_f)):
+        exp_d, exp_f, exp_det = _ieee_expect(fmt, op, dest, srcs)
+        for mode, exp in ((DEST, exp_d), (FLOW, exp_f), (FLOW_DETAIL, exp_f)):
             t = oracle.Table()
             t.scan_records(hdr, arena, mode=mode)
             ents = t.entries()
@@ -207,6 +216,7 @@ def test_bruteforce_ieee_ops(fmt):
             assert got == exp, (op, dest, srcs, mode, got, exp)
             if got is not None:
                 assert int(ents[0]["count"]) == 32
+                assert int(ents[0]["detail"]) == (exp_det if mode == FLOW_DETAIL else 0), (op, srcs, ents)
 
 
 # --------------------------------------------------------------------------
