@@ -207,7 +207,7 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
 fpx_status fpx_scan_records(fpx_handle h, const fpx_rec_hdr* d_hdr, uint64_t n_records, const uint32_t* d_arena,
                             uint64_t arena_planes, uint64_t base_index, uint32_t mode, void* stream) {
   if (!h) return FPX_ERR_INVALID;
-  if (mode != FPX_MODE_DEST && mode != FPX_MODE_FLOW) return FPX_ERR_INVALID;
+  if (mode != FPX_MODE_DEST && mode != FPX_MODE_FLOW && mode != FPX_MODE_FLOW_DETAIL) return FPX_ERR_INVALID;
   if (n_records == 0) return FPX_OK;
   if (!d_hdr || !aligned16(d_hdr)) return FPX_ERR_INVALID;
   if (arena_planes && (!d_arena || !aligned16(d_arena))) return FPX_ERR_INVALID;

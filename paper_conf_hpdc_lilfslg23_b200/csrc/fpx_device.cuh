@@ -88,8 +88,10 @@ __device__ __forceinline__ int dest_kind(uint32_t op, uint32_t fmt, uint32_t lo,
   return kind_of_cls(c);
 }
 
+// code = detail << 4 | flow << 2 | kind  ->  key = site << 32 | detail << 6 | fmt << 4 | flow << 2 | kind
 __device__ __forceinline__ unsigned long long make_key(uint32_t site, uint32_t fmt, uint32_t code) {
-  return ((unsigned long long)site << 32) | ((unsigned long long)fmt << 4) | (unsigned long long)code;
+  return ((unsigned long long)site << 32) | ((unsigned long long)(code >> 4) << 6) | ((unsigned long long)fmt << 4) |
+         (unsigned long long)(code & 15u);
 }
 
 // murmur3 fmix64
@@ -146,6 +148,21 @@ __device__ __forceinline__ void warp_flush(const TableView& tv, uint32_t code_ma
     all &= all - 1;
     const uint32_t tot = __reduce_add_sync(FULL, count_of(c));
     if ((threadIdx.x & 31) == 0) table_add(tv, make_key(site, fmt, (uint32_t)c), tot, gidx);
+  }
+}
+
+// Warp aggregation when every lane holds at most one event code (the FLOW
+// modes): lanes with equal codes are grouped with a ballot per distinct code;
+// the lowest lane of each group updates the table.  Full warp (uniform).
+__device__ __forceinline__ void warp_flush_single(const TableView& tv, int code, uint32_t site, uint32_t fmt,
+                                                  unsigned long long gidx) {
+  uint32_t pending = __ballot_sync(FULL, code >= 0);
+  while (pending) {
+    const int leader = __ffs(pending) - 1;
+    const int c = __shfl_sync(FULL, code, leader);
+    const uint32_t peers = __ballot_sync(FULL, code == c);
+    if ((int)(threadIdx.x & 31) == leader) table_add(tv, make_key(site, fmt, (uint32_t)c), __popc(peers), gidx);
+    pending &= ~peers;
   }
 }
 

@@ -42,7 +42,7 @@ __device__ __forceinline__ bool record_valid(const uint4 h, uint64_t arena_plane
   ok &= !(fmt == FPX_FP64 && (dw & 1u));
   const uint64_t planes = dw + (uint64_t)nsrc_of(meta) * sw_of(fmt);
   ok &= (uint64_t)h.w + planes <= arena_planes;
-  if (MODE == FPX_MODE_FLOW) {
+  if (MODE != FPX_MODE_DEST) {
     ok &= (fmt == FPX_FP32 || fmt == FPX_FP64);
     ok &= (dw == 0u || dw == sw_of(fmt));
   }
@@ -68,7 +68,7 @@ __device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t
   const bool have_div = (op == FPX_OP_DIV) && nsrc >= 2 && dw == sw;
   // destination words d[0..dw) and source words s[0..ns_words) of this lane
   uint32_t ns_words = 0;
-  if (MODE == FPX_MODE_FLOW) ns_words = nsrc * sw;
+  if (MODE != FPX_MODE_DEST) ns_words = nsrc * sw;
   else if (have_div) ns_words = 2 * sw;
   const uint32_t* p = lane_base + (uint64_t)d.val_off * 32;
   uint32_t dv[4], sv[6];
@@ -106,14 +106,16 @@ __device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t
     }
     return cm;
   } else {
-    // Analyzer: S = most severe class among the pre-execution sources.
+    // Analyzer: S = most severe class among the pre-execution sources; src =
+    // the lowest-index source holding it (R21).
     int S = CODE_NONE, sev = 0;
+    uint32_t src = 0;
 #pragma unroll
     for (uint32_t k = 0; k < 3; ++k) {
       if (k >= nsrc) break;
       const uint32_t c = fmt == FPX_FP64 ? cls_fp64(sv[2 * k], sv[2 * k + 1]) : cls_fp32(sv[k]);
       const int sv_ = c == CLS_NAN ? 3 : c == CLS_INF ? 2 : c == CLS_SUB ? 1 : 0;
-      if (sv_ > sev) { sev = sv_; S = kind_of_cls(c); }
+      if (sv_ > sev) { sev = sv_; S = kind_of_cls(c); src = k; }
     }
     int D = CODE_NONE;
     if (dw != 0u) {
@@ -125,9 +127,33 @@ __device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t
     else if (D >= 0) code = (FPX_PROP << 2) | D;
     else if (S >= 0) code = (FPX_KILL << 2) | S;
     if (code < 0) return 0u;
+    // FLOW_DETAIL: detail = 1 + src, | CMP for Table 1's control-flow opcodes (R22)
+    if (MODE == FPX_MODE_FLOW_DETAIL && S >= 0) {
+      const bool cf = op == FPX_OP_FSEL || op == FPX_OP_FSET || op == FPX_OP_FSETP || op == FPX_OP_FMNMX ||
+                      op == FPX_OP_DSETP;
+      code |= (int)((src + 1u) | (cf ? (uint32_t)FPX_DETAIL_CMP : 0u)) << 4;
+    }
     codes = (uint32_t)code;
     evm = 1u;
-    return 1u << code;
+    return 1u;
+  }
+}
+
+// Exact evaluation + warp aggregation + table update of one record.
+template <int MODE>
+__device__ __forceinline__ void flush_record(const RecDesc& d, const uint32_t* __restrict__ lane_base, int lane,
+                                             uint64_t gidx, const TableView& tv) {
+  uint32_t codes, evm;
+  const uint32_t cm = eval_record<MODE>(d, lane_base, lane, codes, evm);
+  if (MODE == FPX_MODE_DEST) {
+    warp_flush(tv, cm, d.site, fmt_of(d.meta), gidx, [&](int c) {
+      uint32_t n = 0;
+#pragma unroll
+      for (int v = 0; v < 8; ++v) n += (((evm >> v) & 1u) && (((codes >> (4 * v)) & 15u) == (uint32_t)c)) ? 1u : 0u;
+      return n;
+    });
+  } else {
+    warp_flush_single(tv, cm ? (int)codes : CODE_NONE, d.site, fmt_of(d.meta), gidx);
   }
 }
 
@@ -138,14 +164,7 @@ __device__ __noinline__ void exact_tile(const RecDesc* __restrict__ recs, const 
     const RecDesc d = recs[j];
     if (d.mask == 0u) continue;  // warp-uniform
     if (MODE == FPX_MODE_DEST && is_compare(op_of(d.meta))) continue;
-    uint32_t codes, evm;
-    const uint32_t cm = eval_record<MODE>(d, lane_base, lane, codes, evm);
-    warp_flush(tv, cm, d.site, fmt_of(d.meta), gidx0 + j, [&](int c) {
-      uint32_t n = 0;
-#pragma unroll
-      for (int v = 0; v < 8; ++v) n += (((evm >> v) & 1u) && (((codes >> (4 * v)) & 15u) == (uint32_t)c)) ? 1u : 0u;
-      return n;
-    });
+    flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv);
   }
 }
 
@@ -164,14 +183,7 @@ __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, 
                     __shfl_sync(FULL, h.x, j)};
     if (d.mask == 0u) continue;  // warp-uniform
     if (MODE == FPX_MODE_DEST && is_compare(op_of(d.meta))) continue;
-    uint32_t codes, evm;
-    const uint32_t cm = eval_record<MODE>(d, lane_base, lane, codes, evm);
-    warp_flush(tv, cm, d.site, fmt_of(d.meta), gidx0 + j, [&](int c) {
-      uint32_t nn = 0;
-#pragma unroll
-      for (int v = 0; v < 8; ++v) nn += (((evm >> v) & 1u) && (((codes >> (4 * v)) & 15u) == (uint32_t)c)) ? 1u : 0u;
-      return nn;
-    });
+    flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv);
   }
 }
 

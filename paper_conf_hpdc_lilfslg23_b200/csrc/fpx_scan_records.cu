@@ -139,7 +139,7 @@ __device__ __forceinline__ uint32_t decode_items(const uint4 h, uint64_t arena_p
   bool v = inrange & (h.x != FPX_SITE_INVALID) & (meta < 0x8000u) & (op < (uint32_t)FPX_OP_COUNT) & (dw <= 4u) &
            !((is64 != 0u) & ((dw & 1u) != 0u));
   v &= (uint64_t)h.w + all_planes <= arena_planes;
-  if (MODE == FPX_MODE_FLOW) v &= (fmt <= 1u) & ((dw == 0u) | (dw == 1u + is64));
+  if (MODE != FPX_MODE_DEST) v &= (fmt <= 1u) & ((dw == 0u) | (dw == 1u + is64));
   ok = v;
   const bool live = v & (h.y != 0u);
   force = live & (op == FPX_OP_DIV);
@@ -617,7 +617,9 @@ cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint
                                 cudaStream_t s) {
   if (mode == FPX_MODE_DEST)
     return launch_records_t<FPX_MODE_DEST>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, s);
-  return launch_records_t<FPX_MODE_FLOW>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, s);
+  if (mode == FPX_MODE_FLOW)
+    return launch_records_t<FPX_MODE_FLOW>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, s);
+  return launch_records_t<FPX_MODE_FLOW_DETAIL>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, s);
 }
 
 }  // namespace fpx

@@ -47,15 +47,20 @@ def detector_lines(entries: np.ndarray, names: dict | None = None) -> list[str]:
 
 
 def analyzer_lines(entries: np.ndarray, names: dict | None = None) -> list[str]:
-    """One line per FLOW entry: the Table 2 state of the instruction site."""
+    """One line per FLOW entry: the Table 2 state of the instruction site; with
+    FPX_MODE_FLOW_DETAIL entries also the Comparison state and the source
+    operand that carried the exceptional value (fn4 P:99)."""
     out = []
     for e in entries:
         flow = int(e["flow"])
         if flow == 0:
             continue
         kernel, loc = _site_label(int(e["site"]), names)
+        det = int(e["detail"]) if "detail" in e.dtype.names else 0
+        state = "COMPARISON/" + STATE_NAMES[flow] if det & 4 else STATE_NAMES[flow]
+        src = f" from source {(det & 3) - 1}" if det & 3 else ""
         out.append(
-            f"#GPU-FPX-ANA {STATE_NAMES[flow]}: {KIND_NAMES[int(e['kind'])]} @ {loc} in [{kernel}]:"
+            f"#GPU-FPX-ANA {state}: {KIND_NAMES[int(e['kind'])]}{src} @ {loc} in [{kernel}]:"
             f"{int(e['site']) & 0xFFFF} [{FMT_NAMES[int(e['fmt'])]}] count={int(e['count'])} "
             f"first={int(e['first_index'])}"
         )

@@ -139,3 +139,16 @@ def test_selective_policy_is_alg3():
     assert p.should_scan("b") and p.num == {"a": 7, "b": 1}
     p = SelectivePolicy(white_list={"a"}, k=2)
     assert [p.should_scan(x) for x in "aabba"] == [True, False, False, False, True]
+
+
+def test_report_detail_states():
+    from paper_conf_hpdc_lilfslg23_b200 import fpx, report
+
+    e = np.zeros(2, dtype=fpx.ENTRY_DTYPE)
+    e["site"] = [1, 2]
+    e["flow"] = [2, 3]
+    e["kind"] = [1, 0]
+    e["detail"] = [2, 5]  # source 1 (fn4: INF flowed from R3); FSEL with a NaN source 0
+    lines = report.analyzer_lines(e)
+    assert lines[0].startswith("#GPU-FPX-ANA PROPAGATION: INF from source 1")
+    assert lines[1].startswith("#GPU-FPX-ANA COMPARISON/DISAPPEARANCE: NaN from source 0")

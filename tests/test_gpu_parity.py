@@ -13,7 +13,7 @@ import pytest
 import fpxgen
 import oracle
 from _records import (
-    BF16, DEST, FLOW, FP16, FP32, FP64, NAN, NONE, OP_FADD, Trace, describe_diff, entries_equal,
+    BF16, DEST, FLOW, FLOW_DETAIL, FP16, FP32, FP64, NAN, NONE, OP_FADD, Trace, describe_diff, entries_equal,
     expected_from_injections, load_worked_cases, np_class, table_dict,
 )
 
@@ -71,7 +71,7 @@ def test_worked_cases_gpu(fpx):
         tr.add_value_record(site=100 + i, opclass=c["opclass"], fmt=c["fmt"], mask=0x8000_F00F, dest_bits=dest,
                             src_bits=[int(s, 16) for s in c["srcs"]])
     hdr, arena = tr.arrays()
-    for mode, key in ((DEST, "expect_dest"), (FLOW, "expect_flow")):
+    for mode, key in ((DEST, "expect_dest"), (FLOW, "expect_flow"), (FLOW_DETAIL, "expect_flow")):
         got, st, _ = gpu_scan(fpx, hdr, arena, base=5, mode=mode)
         assert st == fpx.OK
         assert_same(got, oracle_scan(hdr, arena, 5, mode).entries())
@@ -83,6 +83,8 @@ def test_worked_cases_gpu(fpx):
             else:
                 kind, flow = c[key]
                 assert mine == {(100 + i, c["fmt"], flow, kind): [9, 5 + i]}, c["name"]
+                det = [int(e["detail"]) for e in got if int(e["site"]) == 100 + i]
+                assert det == [c["expect_detail"] if mode == FLOW_DETAIL else 0], c["name"]
 
 
 def _brute_trace():
@@ -100,7 +102,7 @@ def _brute_trace():
 
 
 @pytest.mark.parametrize("variant", [0, 1], ids=["tma", "ldg"])
-@pytest.mark.parametrize("mode", [DEST, FLOW])
+@pytest.mark.parametrize("mode", [DEST, FLOW, FLOW_DETAIL])
 def test_bruteforce_ieee_ops_gpu(fpx, mode, variant):
     hdr, arena = _brute_trace()
     got, st, _ = gpu_scan(fpx, hdr, arena, base=0, mode=mode, flags=variant)
@@ -112,6 +114,7 @@ RECIPES = [
     ("c1", fpxgen.RECIPE_C1, DEST, 100_000, 200),     # config C1 at full size
     ("mix", fpxgen.RECIPE_MIX, DEST, 200_003, 10_000),
     ("flow", fpxgen.RECIPE_FLOW, FLOW, 150_001, 1_000),
+    ("flow_detail", fpxgen.RECIPE_FLOW, FLOW_DETAIL, 150_001, 1_000),
     ("flow_as_dest", fpxgen.RECIPE_FLOW, DEST, 50_017, 1_000),
     ("packed", fpxgen.RECIPE_PACKED, DEST, 120_007, 1_000),
 ]
@@ -129,8 +132,18 @@ def test_synthetic_trace_parity(fpx, name, recipe, mode, n, sites, variant):
     ref = oracle_scan(hdr, arena, base, mode)
     assert st == fpx.OK and stats.bad_records == 0
     assert_same(got, ref.entries())
-    # and the independent closed form of the planted events
-    assert table_dict(got) == expected_from_injections(hdr, inj, base, mode)
+    # and the independent closed form of the planted events (FLOW_DETAIL
+    # splits entries further by source; its (site, fmt, flow, kind) sums match)
+    if mode == FLOW_DETAIL:
+        merged = {}
+        for e in got:
+            k = (int(e["site"]), int(e["fmt"]), int(e["flow"]), int(e["kind"]))
+            c = merged.setdefault(k, [0, 2**64 - 1])
+            c[0] += int(e["count"])
+            c[1] = min(c[1], int(e["first_index"]))
+        assert merged == expected_from_injections(hdr, inj, base, FLOW)
+    else:
+        assert table_dict(got) == expected_from_injections(hdr, inj, base, mode)
 
 
 @pytest.mark.parametrize("variant", [0, 1], ids=["tma", "ldg"])
