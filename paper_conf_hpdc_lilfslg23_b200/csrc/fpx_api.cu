@@ -273,6 +273,7 @@ fpx_status fpx_table_fetch(fpx_handle h, fpx_entry* host_out, uint64_t capacity,
       e.fmt = (uint8_t)((k[i] >> 4) & 3);
       e.flow = (uint8_t)((k[i] >> 2) & 3);
       e.kind = (uint8_t)(k[i] & 3);
+      e.detail = (uint8_t)((k[i] >> 6) & 7);
       e.count = c[i];
       e.first_index = f[i];
       host_out[i] = e;

@@ -113,12 +113,15 @@ def entries_equal(got, exp):
 
 
 def describe_diff(got, exp, limit=8):
-    g = {(int(e["site"]), int(e["fmt"]), int(e["flow"]), int(e["kind"])): (int(e["count"]), int(e["first_index"])) for e in got}
-    x = {(int(e["site"]), int(e["fmt"]), int(e["flow"]), int(e["kind"])): (int(e["count"]), int(e["first_index"])) for e in exp}
+    def k(e):
+        return (int(e["site"]), int(e["fmt"]), int(e["flow"]), int(e["kind"]), int(e["detail"]))
+
+    g = {k(e): (int(e["count"]), int(e["first_index"])) for e in got}
+    x = {k(e): (int(e["count"]), int(e["first_index"])) for e in exp}
     out = []
-    for k in sorted(set(g) | set(x)):
-        if g.get(k) != x.get(k):
-            out.append(f"key(site,fmt,flow,kind)={k}: got {g.get(k)} expected {x.get(k)}")
+    for kk in sorted(set(g) | set(x)):
+        if g.get(kk) != x.get(kk):
+            out.append(f"key(site,fmt,flow,kind,detail)={kk}: got {g.get(kk)} expected {x.get(kk)}")
             if len(out) >= limit:
                 break
     return f"{len(got)} vs {len(exp)} entries; " + "; ".join(out)
