@@ -1,0 +1,45 @@
+"""Small scans of every kernel family for compute-sanitizer (memcheck,
+racecheck, synccheck): DEST / FLOW / FLOW_DETAIL record scans (TMA ring and
+LDG), a storm trace (exact path + table atomics), tensor scans with ragged
+heads / tails, fetch / FETCH_NEW / reset / merge paths."""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import fpxgen  # noqa: E402
+from paper_conf_hpdc_lilfslg23_b200 import fpx  # noqa: E402
+
+dev = torch.device("cuda", 0)
+for recipe, mode in ((fpxgen.RECIPE_MIX, 0), (fpxgen.RECIPE_FLOW, 1), (fpxgen.RECIPE_FLOW, 2), (fpxgen.RECIPE_PACKED, 0)):
+    p = fpxgen.Params(seed=recipe, n_records=20_011, n_sites=300, recipe=recipe)
+    hdr, arena, planes = fpxgen.generate_device(p)
+    _, w = fpxgen.plan_injections(p, 200, flow=recipe == fpxgen.RECIPE_FLOW)
+    fpxgen.apply_device(w, hdr, arena)
+    for flags in (0, fpx.OPT_SCAN_LDG):
+        with fpx.Handle(0, flags=flags) as h:
+            h.scan_records(hdr, arena, mode=mode, arena_planes=planes)
+            e = h.fetch()
+            n = h.fetch_new()
+            k, c, f = h.fetch_device()
+            u = h.unique_device(torch.cat([k, k]))
+            c2, f2 = h.lookup_device(u)
+            h.reset()
+            h.merge_device(k, c, f)
+            assert len(h.fetch()) == len(e) == len(n)
+p = fpxgen.Params(seed=9, n_records=5000, n_sites=20, recipe=fpxgen.RECIPE_STRESS, dense_nan=1.0)
+hdr, arena, planes = fpxgen.generate_device(p)
+with fpx.Handle(0, table_log2_slots=5) as h:
+    h.scan_records(hdr, arena, arena_planes=planes)
+    h.fetch()
+for dt in (torch.float32, torch.float64, torch.float16, torch.bfloat16):
+    x = torch.randn(100_003, device=dev).to(dt)
+    x[::997] = float("nan")
+    with fpx.Handle(0) as h:
+        for a in range(4):
+            h.scan_tensor(x[a: x.numel() - a], site=a)
+        h.fetch()
+torch.cuda.synchronize()
+print("sanitize workload ok")
