@@ -25,12 +25,7 @@ __global__ void k_reset(Slot* slots, uint64_t n, Ctl* ctl) {
     s.pad = 0;
     slots[i] = s;
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    ctl->bad_records = 0;
-    ctl->dropped_events = 0;
-    ctl->newlog_tail = 0;
-    ctl->newlog_overflow = 0;
-  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) *ctl = Ctl{};
 }
 
 __device__ __forceinline__ void clear_slot(Slot* slots, uint64_t i) {
@@ -54,12 +49,7 @@ __global__ void k_reset_touched(const TableView tv, uint64_t slots) {
   }
 }
 
-__global__ void k_reset_ctl(Ctl* ctl) {
-  ctl->bad_records = 0;
-  ctl->dropped_events = 0;
-  ctl->newlog_tail = 0;
-  ctl->newlog_overflow = 0;
-}
+__global__ void k_reset_ctl(Ctl* ctl) { *ctl = Ctl{}; }  // counters and padding (the whole block is copied to the host)
 
 __global__ void k_compact(const Slot* slots, uint64_t n, uint64_t* keys, uint64_t* counts, uint64_t* firsts,
                           unsigned long long* d_n) {
