@@ -276,7 +276,37 @@ fpx_status fpx_table_reset(fpx_handle h, void* stream);
 /* Synchronise and read the sticky counters. */
 fpx_status fpx_get_stats(fpx_handle h, fpx_stats* out);
 
-/* Free everything owned by the handle (synchronises the device first). */
+/* ------------------------------------------------------------------------ */
+/* Shared table across processes / GPUs (SURVEY §5, §8 e alternative)       */
+/* ------------------------------------------------------------------------ */
+/* One device table that scans on other GPUs update in place through CUDA IPC
+ * peer mappings (NVLink / NVSwitch on a B200 box: remote atomicCAS / Add /
+ * Min), so a multi-GPU scan needs no merge step: the home handle's table is
+ * the union.  Events are rare (the fast path never touches the table), so the
+ * remote traffic is a few atomics per exceptional warp-record.
+ *
+ * fpx_table_export: describe the handle's table (slots, new-key log, counters)
+ * as CUDA IPC handles; *out is plain bytes to pass to other processes.
+ * fpx_open_attached: open a handle on `device` (in another process) whose
+ * scans update the exported table.  Attached handles may scan, fetch and read
+ * stats (peer reads); fpx_table_reset is the home handle's job.  Ordering
+ * across processes is the caller's: synchronise the scanning streams and
+ * barrier before the home fetch.  Errors: FPX_ERR_INVALID, FPX_ERR_CUDA (e.g.
+ * no IPC / peer access between the devices). */
+typedef struct {
+  unsigned char ipc[4][64];   /* cudaIpcMemHandle_t: slots, newlog, newlog_slot, ctl */
+  uint32_t table_log2_slots;
+  uint32_t newlog_capacity;
+  int32_t home_device;
+  uint32_t magic;             /* FPX_IPC_MAGIC */
+} fpx_ipc_table;
+#define FPX_IPC_MAGIC 0x46505831u /* "FPX1" */
+
+fpx_status fpx_table_export(fpx_handle h, fpx_ipc_table* out);
+fpx_status fpx_open_attached(int device, const fpx_ipc_table* table, fpx_handle* out);
+
+/* Free everything owned by the handle (synchronises the device first).  An
+ * attached handle unmaps the shared table; the home handle frees it. */
 fpx_status fpx_close(fpx_handle h);
 
 /* Static string for a status code. */

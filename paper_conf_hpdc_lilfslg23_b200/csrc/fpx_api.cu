@@ -15,6 +15,7 @@ using namespace fpx;
 
 struct fpx_ctx {
   int device = 0;
+  bool attached = false;  // table mapped from another process (fpx_open_attached)
   int num_sms = 148;
   uint32_t variant = 0;  // record-scan kernel: 0 TMA ring, 1 LDG (ablation)
   uint64_t slots = 0;
@@ -359,7 +360,7 @@ fpx_status fpx_table_merge_device(fpx_handle h, const uint64_t* d_keys, const ui
 }
 
 fpx_status fpx_table_reset(fpx_handle h, void* stream) {
-  if (!h) return FPX_ERR_INVALID;
+  if (!h || h->attached) return FPX_ERR_INVALID;  // the home handle owns the shared table
   DeviceGuard g(h->device);
   if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -383,15 +384,84 @@ fpx_status fpx_get_stats(fpx_handle h, fpx_stats* out) {
   return FPX_OK;
 }
 
+fpx_status fpx_table_export(fpx_handle h, fpx_ipc_table* out) {
+  if (!h || !out || h->attached) return FPX_ERR_INVALID;
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  std::memset(out, 0, sizeof *out);
+  void* bases[4] = {h->tv.slots, h->tv.newlog, h->tv.newlog_slot, h->tv.ctl};
+  for (int i = 0; i < 4; ++i) {
+    cudaIpcMemHandle_t m;
+    CK(cudaIpcGetMemHandle(&m, bases[i]));
+    static_assert(sizeof(m) == 64, "cudaIpcMemHandle_t is 64 bytes");
+    std::memcpy(out->ipc[i], &m, sizeof m);
+  }
+  uint32_t lg = 0;
+  while ((1ull << lg) < h->slots) ++lg;
+  out->table_log2_slots = lg;
+  out->newlog_capacity = (uint32_t)h->tv.newlog_cap;
+  out->home_device = h->device;
+  out->magic = FPX_IPC_MAGIC;
+  return FPX_OK;
+}
+
+fpx_status fpx_open_attached(int device, const fpx_ipc_table* t, fpx_handle* out) {
+  if (!out || !t || t->magic != FPX_IPC_MAGIC) return FPX_ERR_INVALID;
+  if (t->table_log2_slots < 4 || t->table_log2_slots > 30 || t->newlog_capacity == 0) return FPX_ERR_INVALID;
+  *out = nullptr;
+  int ndev = 0;
+  CK(cudaGetDeviceCount(&ndev));
+  if (device < 0 || device >= ndev) return FPX_ERR_INVALID;
+  DeviceGuard g(device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  fpx_ctx* h = new (std::nothrow) fpx_ctx();
+  if (!h) return FPX_ERR_NOMEM;
+  h->device = device;
+  h->attached = true;
+  CK(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, device));
+  h->slots = 1ull << t->table_log2_slots;
+  void* ptrs[4] = {nullptr, nullptr, nullptr, nullptr};
+  for (int i = 0; i < 4; ++i) {
+    cudaIpcMemHandle_t m;
+    std::memcpy(&m, t->ipc[i], sizeof m);
+    cudaError_t e = cudaIpcOpenMemHandle(&ptrs[i], m, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+      for (int j = 0; j < i; ++j) cudaIpcCloseMemHandle(ptrs[j]);
+      delete h;
+      return cuda_err(e, "cudaIpcOpenMemHandle");
+    }
+  }
+  h->tv.slots = static_cast<Slot*>(ptrs[0]);
+  h->tv.mask = h->slots - 1;
+  h->tv.newlog = static_cast<unsigned long long*>(ptrs[1]);
+  h->tv.newlog_slot = static_cast<unsigned int*>(ptrs[2]);
+  h->tv.ctl = static_cast<Ctl*>(ptrs[3]);
+  h->tv.newlog_cap = t->newlog_capacity;
+  if (cudaMallocHost(&h->h_ctl, sizeof(Ctl)) != cudaSuccess) {
+    for (int j = 0; j < 4; ++j) cudaIpcCloseMemHandle(ptrs[j]);
+    delete h;
+    return FPX_ERR_NOMEM;
+  }
+  *out = h;
+  return FPX_OK;
+}
+
 fpx_status fpx_close(fpx_handle h) {
   if (!h) return FPX_ERR_INVALID;
   {
     DeviceGuard g(h->device);
     cudaDeviceSynchronize();
-    cudaFree(h->tv.slots);
-    cudaFree(h->tv.newlog);
-    cudaFree(h->tv.newlog_slot);
-    cudaFree(h->tv.ctl);
+    if (h->attached) {
+      cudaIpcCloseMemHandle(h->tv.slots);
+      cudaIpcCloseMemHandle(h->tv.newlog);
+      cudaIpcCloseMemHandle(h->tv.newlog_slot);
+      cudaIpcCloseMemHandle(h->tv.ctl);
+    } else {
+      cudaFree(h->tv.slots);
+      cudaFree(h->tv.newlog);
+      cudaFree(h->tv.newlog_slot);
+      cudaFree(h->tv.ctl);
+    }
     cudaFreeHost(h->h_ctl);
     for (void* p : {(void*)h->d_keys, (void*)h->d_counts, (void*)h->d_first, (void*)h->d_keys2, (void*)h->d_idx,
                     (void*)h->d_idx2, (void*)h->d_n, h->d_temp})

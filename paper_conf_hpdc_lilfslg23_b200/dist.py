@@ -80,3 +80,52 @@ def merge_handle(handle, group=None, stream=None):
     """Fetch this rank's table on device and merge it across the group (NCCL)."""
     k, c, f = handle.fetch_device(stream=stream)
     return merge(k, c, f, DeviceOps(handle, stream), group=group)
+
+
+class SharedTable:
+    """Fused alternative to `merge` (SURVEY §8 e, NEXT): every rank scans into
+    the home rank's device table through CUDA IPC peer mappings — the table
+    updates (rare atomicCAS / Add / Min, only on exceptional warp-records) go
+    over NVLink / NVSwitch inside the scan kernels, so there is no merge step.
+
+        st = SharedTable(device)          # collective: home exports, others attach
+        st.handle.scan_records(...)       # every rank, its own shard
+        st.finish()                       # streams drained + barrier
+        entries = st.fetch()              # home rank: the union table
+    """
+
+    def __init__(self, device: int, group=None, home: int = 0, **handle_kw):
+        from . import fpx
+
+        self.group, self.home = group, home
+        self.rank = dist.get_rank(group)
+        blob = [None]
+        if self.rank == home:
+            self.handle = fpx.Handle(device, **handle_kw)
+            blob = [self.handle.export()]
+        dist.broadcast_object_list(blob, src=home, group=group)
+        if self.rank != home:
+            self.handle = fpx.Handle.attach(device, blob[0])
+
+    def reset(self, stream=None):
+        """Home clears the table; everyone waits for it before scanning again."""
+        if self.rank == self.home:
+            self.handle.reset(stream=stream)
+            torch.cuda.current_stream().synchronize() if stream is None else stream.synchronize()
+        dist.barrier(group=self.group)
+
+    def finish(self, stream=None):
+        (torch.cuda.current_stream() if stream is None else stream).synchronize()
+        dist.barrier(group=self.group)
+
+    def fetch(self):
+        assert self.rank == self.home, "the home rank owns the shared table"
+        return self.handle.fetch()
+
+    def close(self):
+        dist.barrier(group=self.group)  # attached ranks unmap before the home frees
+        if self.rank != self.home:
+            self.handle.close()
+        dist.barrier(group=self.group)
+        if self.rank == self.home:
+            self.handle.close()

@@ -38,6 +38,11 @@ ENTRY_DTYPE = np.dtype(
 HDR_DTYPE = np.dtype([("site", "<u4"), ("active_mask", "<u4"), ("meta", "<u4"), ("val_off", "<u4")])
 
 
+class IpcTable(ctypes.Structure):
+    _fields_ = [("ipc", (ctypes.c_ubyte * 64) * 4), ("table_log2_slots", ctypes.c_uint32),
+                ("newlog_capacity", ctypes.c_uint32), ("home_device", ctypes.c_int32), ("magic", ctypes.c_uint32)]
+
+
 class Options(ctypes.Structure):
     _fields_ = [("table_log2_slots", ctypes.c_uint32), ("newlog_capacity", ctypes.c_uint32),
                 ("flags", ctypes.c_uint32)]
@@ -61,6 +66,8 @@ _SIGS = {
     "fpx_table_merge_device": ([_vp, _vp, _vp, _vp, _u64, _vp], _st),
     "fpx_table_reset": ([_vp, _vp], _st),
     "fpx_get_stats": ([_vp, ctypes.POINTER(Stats)], _st),
+    "fpx_table_export": ([_vp, ctypes.POINTER(IpcTable)], _st),
+    "fpx_open_attached": ([ctypes.c_int, ctypes.POINTER(IpcTable), ctypes.POINTER(_vp)], _st),
     "fpx_close": ([_vp], _st),
     "fpx_strerror": ([_st], ctypes.c_char_p),
     "fpx_last_cuda_error": ([], ctypes.c_char_p),
@@ -130,6 +137,24 @@ class Handle:
     @property
     def ptr(self):
         return self._h
+
+    def export(self) -> bytes:
+        """The table as CUDA IPC handles (fpx_table_export), for attach()."""
+        t = IpcTable()
+        check(lib.fpx_table_export(self._h, ctypes.byref(t)), "fpx_table_export")
+        return bytes(t)
+
+    @classmethod
+    def attach(cls, device: int, exported: bytes) -> "Handle":
+        """A handle on `device` (in another process) whose scans update the
+        exported table in place through peer memory (fpx_open_attached)."""
+        self = cls.__new__(cls)
+        self._h = _vp()
+        t = IpcTable.from_buffer_copy(exported)
+        check(lib.fpx_open_attached(device, ctypes.byref(t), ctypes.byref(self._h)), "fpx_open_attached")
+        self.device = device
+        self.last_status = OK
+        return self
 
     def scan_records(self, hdr, arena, base_index: int = 0, mode: int = MODE_DEST, stream=None, n_records=None,
                      arena_planes=None):

@@ -121,3 +121,61 @@ def test_two_rank_merge_on_device_ops():
     for rank, k, c, f in res:
         assert dict(zip(k, zip(c, f))) == ref, rank
         assert k == sorted(k, key=lambda x: x % (1 << 64))  # ascending uint64 key order
+
+
+def _rank_shared(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_hpdc_lilfslg23_b200 import dist as fdist
+
+    n = 1_000_003
+    p = fpxgen.Params(seed=6, n_records=n, n_sites=2000, recipe=fpxgen.RECIPE_FLOW, p_fp64=0.3)
+    hdr, arena, planes = fpxgen.generate_device(p)
+    _, w = fpxgen.plan_injections(p, 2000, flow=True)
+    fpxgen.apply_device(w, hdr, arena)
+    a, b = fdist.shard_range(n, rank, world)
+    st = fdist.SharedTable(0)
+    for rep in range(2):  # the second pass exercises the shared reset
+        st.reset()
+        st.handle.scan_records(hdr[a:b], arena, base_index=a, arena_planes=planes, mode=1)
+        st.finish()
+        if rank == 0:
+            ents = st.fetch()
+            q.put((rep, ents.tobytes()))
+    st.close()
+    dist.destroy_process_group()
+
+
+def test_shared_table_across_processes():
+    """Two processes (here sharing cuda:0; on an 8-GPU box each its own GPU,
+    peer-mapped over NVLink) scan their shards straight into rank 0's table."""
+    import torch.multiprocessing as mp
+
+    from paper_conf_hpdc_lilfslg23_b200 import fpx
+
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rank_shared, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    res = [q.get(timeout=300) for _ in range(2)]
+    for pr in procs:
+        pr.join(timeout=120)
+        assert pr.exitcode == 0
+    n = 1_000_003
+    p = fpxgen.Params(seed=6, n_records=n, n_sites=2000, recipe=fpxgen.RECIPE_FLOW, p_fp64=0.3)
+    hdr, arena = fpxgen.generate_host(p)
+    _, w = fpxgen.plan_injections(p, 2000, flow=True)
+    fpxgen.apply_host(w, hdr, arena)
+    t = oracle.Table()
+    t.scan_records(hdr, arena, mode=1)
+    exp = t.entries()
+    for rep, blob in res:
+        got = np.frombuffer(blob, dtype=fpx.ENTRY_DTYPE)
+        assert entries_equal(got, exp), (rep, describe_diff(got, exp))
