@@ -378,6 +378,10 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--variant", default="tma", choices=["tma", "ldg"], help="record-scan kernel (ldg = ablation)")
+    ap.add_argument("--debug-one-gpu", action="store_true",
+                    help="testing only: every rank on cuda:0 with gloo (exercises the N > 1 code paths on one GPU)")
+    ap.add_argument("--merge", default="nccl", choices=["nccl", "peer"],
+                    help="N > 1: NCCL merge of per-GPU tables, or one shared table updated over NVLink peer memory")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     cfg = dict(CONFIGS[args.config])
@@ -398,8 +402,12 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     assert world == args.gpus or world == 1, "launch N>1 with torchrun"
+    if args.debug_one_gpu:
+        local = 0
     torch.cuda.set_device(local)
-    if world > 1:
+    if world > 1 and args.debug_one_gpu:
+        dist.init_process_group("gloo")
+    elif world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
 
@@ -411,14 +419,25 @@ def main():
         wl = RecordsWorkload(cfg, rank, seed, args.variant)
     torch.cuda.synchronize()
 
+    shared = None
+    if world > 1 and args.merge == "peer":
+        h.close()
+        shared = fdist.SharedTable(local, flags=fpx.OPT_SCAN_LDG if args.variant == "ldg" else 0)
+        h = shared.handle
+
     def step(ev_a=None, ev_b=None):
-        h.reset(stream=stream)
+        if shared is not None:
+            shared.reset(stream=stream)  # home clears; everyone waits
+        else:
+            h.reset(stream=stream)
         if ev_a is not None:
             ev_a.record(stream)
         wl.scan(h, stream)
         if ev_b is not None:
             ev_b.record(stream)
-        if world > 1:
+        if shared is not None:
+            shared.finish(stream=stream)  # every rank's inserts landed in the home table
+        elif world > 1:
             fdist.merge_handle(h, stream=stream)
 
     for _ in range(args.warmup):
@@ -444,13 +463,17 @@ def main():
     total_ms = t_start.elapsed_time(t_end)
     kern_ms = float(np.mean([a.elapsed_time(b) for a, b in evs]))
     if world > 1:
-        t = torch.tensor([total_ms, kern_ms], dtype=torch.float64, device=dev)
+        tdev = torch.device("cpu") if dist.get_backend() == "gloo" else dev
+        t = torch.tensor([total_ms, kern_ms], dtype=torch.float64, device=tdev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms, kern_ms = float(t[0]), float(t[1])
     ms_per_step = total_ms / K
 
-    ents = h.fetch()
-    ok_status = h.last_status
+    if shared is None or rank == 0:
+        ents = h.fetch()
+        ok_status = h.last_status
+    else:
+        ents, ok_status = [], 0
 
     # e2e: the same metric through the public API with host buffers: per step,
     # H2D of the step's inputs from pinned memory, scan, fetch (D2H of entries)
@@ -482,6 +505,8 @@ def main():
     lane_values, nbytes = wl.lane_values, wl.nbytes
 
     if rank != 0:
+        if shared is not None:
+            shared.close()
         if world > 1:
             dist.destroy_process_group()
         return 0
@@ -495,7 +520,7 @@ def main():
             tj = json.load(f)
         traffic = tj.get(args.config, {}).get("dram_bytes_per_launch")
     clocks = clk.summary()
-    cpu = None if args.no_cpu_baseline else wl.cpu_baseline()
+    cpu = None if (args.no_cpu_baseline or world > 1) else wl.cpu_baseline()  # rank 0 at N = 1 only
     line = {
         "metric": METRIC,
         "value": world * lane_values / (ms_per_step / 1e3),
@@ -517,7 +542,9 @@ def main():
             "table_entries": int(len(ents)),
             "fetch_status": int(ok_status),
             "l2": "inputs >> 126 MB L2 (no flush needed)",
-            "parallelism": f"shards x{world}" + (" + NCCL merge per step" if world > 1 else ""),
+            "parallelism": f"shards x{world}" + ("" if world == 1 else (" + shared table over NVLink peer memory"
+                                                                         if shared is not None else
+                                                                         " + NCCL merge per step")),
         },
         "roofline": {
             "bound": "hbm",
@@ -534,12 +561,15 @@ def main():
         # per step: table reset (2 kernels) + scan (1); merge (N > 1): compact, iota,
         # radix sort, gather, sort, select-init, select, lookup (counted with ncu,
         # tools/count_merge_launches.py); NCCL's own kernels are not ours
-        "gpu_launches": K * (3 + (8 if world > 1 else 0)),
+        "gpu_launches": K * (3 + (8 if (world > 1 and shared is None) else 0)),
         "cpu_baseline": cpu,
         "e2e": e2e,
     }
     print(json.dumps(line), flush=True)
-    h.close()
+    if shared is not None:
+        shared.close()
+    else:
+        h.close()
     if world > 1:
         dist.destroy_process_group()
     return 0
