@@ -380,7 +380,7 @@ def main():
     ap.add_argument("--variant", default="tma", choices=["tma", "ldg"], help="record-scan kernel (ldg = ablation)")
     ap.add_argument("--debug-one-gpu", action="store_true",
                     help="testing only: every rank on cuda:0 with gloo (exercises the N > 1 code paths on one GPU)")
-    ap.add_argument("--merge", default="nccl", choices=["nccl", "peer"],
+    ap.add_argument("--merge", default="peer", choices=["nccl", "peer"],
                     help="N > 1: NCCL merge of per-GPU tables, or one shared table updated over NVLink peer memory")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
@@ -419,11 +419,15 @@ def main():
         wl = RecordsWorkload(cfg, rank, seed, args.variant)
     torch.cuda.synchronize()
 
-    shared = None
+    shared, merge_note = None, None
     if world > 1 and args.merge == "peer":
-        h.close()
-        shared = fdist.SharedTable(local, flags=fpx.OPT_SCAN_LDG if args.variant == "ldg" else 0)
-        h = shared.handle
+        try:
+            shared = fdist.SharedTable(local, flags=fpx.OPT_SCAN_LDG if args.variant == "ldg" else 0)
+            h.close()
+            h = shared.handle
+        except RuntimeError as ex:  # no peer / IPC access: fall back to the NCCL merge, and say so
+            merge_note = f"peer table unavailable ({str(ex)[:120]}); NCCL merge used"
+    merged = [None]
 
     def step(ev_a=None, ev_b=None):
         if shared is not None:
@@ -438,7 +442,7 @@ def main():
         if shared is not None:
             shared.finish(stream=stream)  # every rank's inserts landed in the home table
         elif world > 1:
-            fdist.merge_handle(h, stream=stream)
+            merged[0] = fdist.merge_handle(h, stream=stream)
 
     for _ in range(args.warmup):
         step()
@@ -474,10 +478,14 @@ def main():
         ok_status = h.last_status
     else:
         ents, ok_status = [], 0
+    if merged[0] is not None:  # NCCL merge: report the merged (global) table
+        ents = merged[0][0]
 
     # e2e: the same metric through the public API with host buffers: per step,
     # H2D of the step's inputs from pinned memory, scan, fetch (D2H of entries)
     e2e = None
+    if world > 1:
+        e2e = {"value": None, "unit": UNIT, "reason": "e2e (host buffers) is measured at N = 1 only"}
     if not args.no_e2e and world == 1:
         try:
             wl.make_host_copies()
@@ -545,6 +553,7 @@ def main():
             "parallelism": f"shards x{world}" + ("" if world == 1 else (" + shared table over NVLink peer memory"
                                                                          if shared is not None else
                                                                          " + NCCL merge per step")),
+            **({"merge_note": merge_note} if merge_note else {}),
         },
         "roofline": {
             "bound": "hbm",

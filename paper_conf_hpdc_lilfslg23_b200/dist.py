@@ -104,8 +104,23 @@ class SharedTable:
             self.handle = fpx.Handle(device, **handle_kw)
             blob = [self.handle.export()]
         dist.broadcast_object_list(blob, src=home, group=group)
+        err = None
         if self.rank != home:
-            self.handle = fpx.Handle.attach(device, blob[0])
+            try:
+                self.handle = fpx.Handle.attach(device, blob[0])
+            except fpx.FpxError as e:  # e.g. no IPC / peer access between the GPUs
+                self.handle, err = None, str(e)
+        # collective verdict: every rank must be attached, else nobody uses it
+        flags = [None] * dist.get_world_size(group)
+        dist.all_gather_object(flags, err, group=group)
+        self.error = next((f for f in flags if f is not None), None)
+        if self.error is not None:
+            if self.handle is not None and self.rank != home:
+                self.handle.close()
+            dist.barrier(group=group)
+            if self.rank == home:
+                self.handle.close()
+            raise RuntimeError(f"shared table unavailable: {self.error}")
 
     def reset(self, stream=None):
         """Home clears the table; everyone waits for it before scanning again."""
