@@ -368,3 +368,28 @@ def test_reset_clears_every_key(fpx, newlog_capacity):
             assert st.newlog_overflow == (0 if newlog_capacity == 0 else len(ref) - newlog_capacity)
             h.reset()
             assert len(h.fetch()) == 0 and h.stats().table_entries == 0
+
+
+@pytest.mark.parametrize("mode", [DEST, FLOW, FLOW_DETAIL])
+def test_irregular_layouts(fpx, mode):
+    """Producer layouts the generator never makes: records in shuffled arena
+    order, several records sharing planes (broadcast immediates),
+    records whose planes run past the arena (bad), DEST scans of records with
+    sources (needed planes stop before the footprint ends)."""
+    p = fpxgen.Params(seed=17, n_records=40_000, n_sites=300, recipe=fpxgen.RECIPE_FLOW, p_fp64=0.4)
+    hdr, arena = fpxgen.generate_host(p)
+    _, w = fpxgen.plan_injections(p, 400, flow=True)
+    fpxgen.apply_host(w, hdr, arena)
+    rng = np.random.default_rng(5)
+    hdr2 = hdr.copy()
+    perm = rng.permutation(len(hdr2))
+    hdr2 = hdr2[perm]                                         # records no longer in arena order
+    share = rng.choice(len(hdr2), 2000, replace=False)
+    hdr2["val_off"][share[1000:]] = hdr2["val_off"][share[:1000]]  # pairs of records share planes
+    hdr2["meta"][share[1000:]] = hdr2["meta"][share[:1000]]
+    oob = rng.choice(len(hdr2), 50, replace=False)
+    hdr2["val_off"][oob] = arena.shape[0] - 1                 # planes past the arena end -> bad records
+    got, st, stats = gpu_scan(fpx, hdr2, arena, base=77, mode=mode)
+    ref = oracle_scan(hdr2, arena, 77, mode)
+    assert_same(got, ref.entries())
+    assert stats.bad_records == ref.bad_records > 0
