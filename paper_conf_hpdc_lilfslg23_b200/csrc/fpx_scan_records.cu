@@ -221,7 +221,10 @@ __device__ __forceinline__ uint4 and4(uint4 a, uint4 b) { return make_uint4(a.x 
 template <uint32_t FMT, bool PARTIAL>
 __device__ __forceinline__ void consume_list(Witness& w, uint32_t b, uint32_t e, uint32_t items_addr,
                                              uint32_t planes_addr, uint32_t g, uint32_t q) {
-#pragma unroll 2
+#ifndef FPX_CONSUME_UNROLL
+#define FPX_CONSUME_UNROLL 2
+#endif
+#pragma unroll FPX_CONSUME_UNROLL
   for (uint32_t i = b + g; i < e; i += 4) {
     const uint2 it = lds64(items_addr + i * 8);
     const uint32_t a = planes_addr + it.x * 128 + q * 16;

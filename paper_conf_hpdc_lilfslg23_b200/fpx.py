@@ -15,7 +15,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_LIB_PATH = os.path.join(_HERE, "libfpx.so")
+_LIB_PATH = os.environ.get("FPX_LIB") or os.path.join(_HERE, "libfpx.so")  # FPX_LIB: A/B builds (tuning)
 if not os.path.exists(_LIB_PATH):
     raise ImportError(f"{_LIB_PATH} is missing: build it with `python __graft_entry__.py build` (no CPU fallback)")
 lib = ctypes.CDLL(_LIB_PATH)
