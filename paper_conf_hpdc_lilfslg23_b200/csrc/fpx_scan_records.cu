@@ -214,6 +214,11 @@ __device__ __forceinline__ uint4 quad_ext(uint32_t mask, uint32_t q) {
 }
 __device__ __forceinline__ uint4 and4(uint4 a, uint4 b) { return make_uint4(a.x & b.x, a.y & b.y, a.z & b.z, a.w & b.w); }
 
+#ifndef FPX_CONSUME_UNROLL
+#define FPX_CONSUME_UNROLL 2
+#endif
+constexpr int kConsumeUnroll = FPX_CONSUME_UNROLL;
+
 // Consume one item list with the lane-quad layout: thread (g = lane / 8,
 // q = lane % 8) reads words 4q..4q+3 (lanes 4q..4q+3 of the instrumented
 // warp) of item i + g, so one warp step covers four items with one 128-bit
@@ -221,10 +226,7 @@ __device__ __forceinline__ uint4 and4(uint4 a, uint4 b) { return make_uint4(a.x 
 template <uint32_t FMT, bool PARTIAL>
 __device__ __forceinline__ void consume_list(Witness& w, uint32_t b, uint32_t e, uint32_t items_addr,
                                              uint32_t planes_addr, uint32_t g, uint32_t q) {
-#ifndef FPX_CONSUME_UNROLL
-#define FPX_CONSUME_UNROLL 2
-#endif
-#pragma unroll FPX_CONSUME_UNROLL
+#pragma unroll kConsumeUnroll
   for (uint32_t i = b + g; i < e; i += 4) {
     const uint2 it = lds64(items_addr + i * 8);
     const uint32_t a = planes_addr + it.x * 128 + q * 16;
