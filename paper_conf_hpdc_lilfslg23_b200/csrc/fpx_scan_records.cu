@@ -215,7 +215,7 @@ __device__ __forceinline__ uint4 quad_ext(uint32_t mask, uint32_t q) {
 __device__ __forceinline__ uint4 and4(uint4 a, uint4 b) { return make_uint4(a.x & b.x, a.y & b.y, a.z & b.z, a.w & b.w); }
 
 #ifndef FPX_CONSUME_UNROLL
-#define FPX_CONSUME_UNROLL 2
+#define FPX_CONSUME_UNROLL 1  // A/B on B200 (tools/ab.sh): 1 beats 2 and 4 by 2-5 %
 #endif
 constexpr int kConsumeUnroll = FPX_CONSUME_UNROLL;
 
