@@ -414,8 +414,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 // one, default RING_DEFAULT.
 using Ring0 = RingCfg<16, 2, 52>;
 using Ring1 = RingCfg<20, 2, 40>;
-using Ring2 = RingCfg<16, 3, 32>;
-using Ring3 = RingCfg<18, 2, 46>;
+using Ring2 = RingCfg<22, 2, 36>;
+using Ring3 = RingCfg<24, 2, 32>;
 static_assert(sizeof(WarpSmem<Ring2>) % 128 == 0 && ring_smem<Ring0>() <= 227 * 1024 && ring_smem<Ring1>() <= 227 * 1024 &&
                   ring_smem<Ring2>() <= 227 * 1024 && ring_smem<Ring3>() <= 227 * 1024,
               "ring exceeds shared memory");
@@ -595,9 +595,11 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
                                                                          d_arena, arena_planes, base_index, tv);
     return cudaGetLastError();
   }
-  // Ring geometry: big stages pay off when records carry several planes (per
-  // tile fixed work is amortised over more bytes), more warps when they carry
-  // about one (C5-like FP32 traces).  Estimated from the arena density;
+  // Ring geometry, from interleaved A/B runs on B200 (tools/ab_env.sh,
+  // profiles/r1/ab_rings.txt): 20 warps x 2 stages x 40 planes for traces
+  // with several planes per record (C2, C3, C4a); 24 x 2 x 32 when records
+  // carry about one plane (C5-like FP32 traces, estimated from the arena
+  // density).  Warp counts stay multiples of 4 (one share per SM sub-partition).
   // FPX_RING (environment, tuning only) overrides.
   static int forced = -2;
   if (forced == -2) {
@@ -605,7 +607,7 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
     forced = e ? atoi(e) : -1;
   }
   int ring = forced;
-  if (ring < 0) ring = (arena_planes * 4 < n * 5) ? 1 : 0;  // < 1.25 planes per record -> 20-warp ring
+  if (ring < 0) ring = (arena_planes * 4 < n * 5) ? 3 : 1;  // < 1.25 planes per record
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   switch (ring) {
     case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
