@@ -414,7 +414,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 // one, default RING_DEFAULT.
 using Ring0 = RingCfg<16, 2, 52>;
 using Ring1 = RingCfg<20, 2, 40>;
-using Ring2 = RingCfg<22, 2, 36>;
+using Ring2 = RingCfg<28, 2, 28>;
 using Ring3 = RingCfg<24, 2, 32>;
 static_assert(sizeof(WarpSmem<Ring2>) % 128 == 0 && ring_smem<Ring0>() <= 227 * 1024 && ring_smem<Ring1>() <= 227 * 1024 &&
                   ring_smem<Ring2>() <= 227 * 1024 && ring_smem<Ring3>() <= 227 * 1024,
