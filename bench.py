@@ -45,6 +45,10 @@ CONFIGS = {
     "c4b": dict(name="C4b: fpx_scan_tensor over 40 GB of BF16 model activations (2e10 torch.randn values), "
                      "sparse NaN/INF at 1e-7 plus whole-row NaN bursts",
                 kind="tensor", n=20_000_000_000, dtype="bf16", rho=1e-7, sites=1, mode=0, recipe=-1, p_fp64=0.0),
+    "s1": dict(name="S (stress): 1e7 FP32 FFMA records over 200 sites, every active lane NaN (rho = 1)",
+               recipe=4, n=10_000_000, sites=200, p_fp64=0.0, mode=0, n_inj=0, dense=1.0),
+    "s2": dict(name="S (stress): 1e7 FP32 FFMA records over 200 sites, NaN density 1e-2",
+               recipe=4, n=10_000_000, sites=200, p_fp64=0.0, mode=0, n_inj=0, dense=0.01),
     "c5": dict(name="C5 shard: FP32 dest-only trace, 10^11 lane-values / 8 GPUs = 3.9e8 records per GPU, 1e6 sites",
                recipe=1, n=390_625_000, sites=1_000_000, p_fp64=0.0, mode=0, rho=1e-6),
 }
@@ -139,9 +143,10 @@ def build_trace(cfg, rank, world, seed):
 
     n = cfg["n"]
     r0 = rank * n
-    p = fpxgen.Params(seed=seed, n_records=n, n_sites=cfg["sites"], recipe=cfg["recipe"], p_fp64=cfg["p_fp64"])
+    p = fpxgen.Params(seed=seed, n_records=n, n_sites=cfg["sites"], recipe=cfg["recipe"], p_fp64=cfg["p_fp64"],
+                      dense_nan=cfg.get("dense", 0.0))
     hdr, arena, planes = fpxgen.generate_device(p, r0=r0)
-    n_inj = cfg.get("n_inj") or int(round(cfg["rho"] * n * 32))
+    n_inj = cfg["n_inj"] if "n_inj" in cfg else int(round(cfg["rho"] * n * 32))
     inj, writes = fpxgen.plan_injections(p, n_inj, flow=cfg["mode"] == 1, r0=r0)
     fpxgen.apply_device(writes, hdr, arena)
     return p, hdr, arena, planes, r0, inj

@@ -136,32 +136,62 @@ static __device__ __noinline__ void table_add(const TableView tv, unsigned long 
   atomicAdd(&tv.ctl->dropped_events, cnt);
 }
 
+// Table updates of one warp, batched: the warp-reduced (key, count, first)
+// events of a tile are parked one per lane and issued by up to 32 lanes at
+// once, so a dense tile (storms) costs ~one L2 round trip per 32 events
+// instead of one per event.  Consecutive events with the same key (a storm
+// over one site) merge before any atomic.  `n` and `last` are warp-uniform.
+struct PendingEvents {
+  unsigned long long key = 0, first = 0, last = FPX_KEY_EMPTY;
+  uint32_t count = 0, n = 0;
+  __device__ __forceinline__ void push(const TableView& tv, unsigned long long k, uint32_t c,
+                                       unsigned long long f) {
+    const uint32_t lane = threadIdx.x & 31;
+    if (n != 0 && k == last) {  // same key as the previous event: merge (first is already the smaller)
+      if (lane == n - 1) count += c;
+      return;
+    }
+    if (lane == n) {
+      key = k;
+      count = c;
+      first = f;
+    }
+    last = k;
+    if (++n == 32) flush(tv);
+  }
+  __device__ __forceinline__ void flush(const TableView& tv) {
+    if ((threadIdx.x & 31) < n) table_add(tv, key, count, first);
+    n = 0;
+    last = FPX_KEY_EMPTY;
+    __syncwarp();
+  }
+};
+
 // Warp aggregation of one record's events.  Every lane passes a bitmask of
 // the codes it holds (bit c = code c present) plus, per code, its count via
 // the `count_of` functor.  Must be called by the full warp (uniform).
 template <typename CountOf>
-__device__ __forceinline__ void warp_flush(const TableView& tv, uint32_t code_mask, uint32_t site, uint32_t fmt,
-                                           unsigned long long gidx, CountOf count_of) {
+__device__ __forceinline__ void warp_flush(const TableView& tv, PendingEvents& pend, uint32_t code_mask,
+                                           uint32_t site, uint32_t fmt, unsigned long long gidx, CountOf count_of) {
   uint32_t all = __reduce_or_sync(FULL, code_mask);
   while (all) {
     const int c = __ffs(all) - 1;
     all &= all - 1;
     const uint32_t tot = __reduce_add_sync(FULL, count_of(c));
-    if ((threadIdx.x & 31) == 0) table_add(tv, make_key(site, fmt, (uint32_t)c), tot, gidx);
+    pend.push(tv, make_key(site, fmt, (uint32_t)c), tot, gidx);
   }
 }
 
 // Warp aggregation when every lane holds at most one event code (the FLOW
-// modes): lanes with equal codes are grouped with a ballot per distinct code;
-// the lowest lane of each group updates the table.  Full warp (uniform).
-__device__ __forceinline__ void warp_flush_single(const TableView& tv, int code, uint32_t site, uint32_t fmt,
-                                                  unsigned long long gidx) {
+// modes): lanes with equal codes are grouped with a ballot per distinct code.
+__device__ __forceinline__ void warp_flush_single(const TableView& tv, PendingEvents& pend, int code, uint32_t site,
+                                                  uint32_t fmt, unsigned long long gidx) {
   uint32_t pending = __ballot_sync(FULL, code >= 0);
   while (pending) {
     const int leader = __ffs(pending) - 1;
     const int c = __shfl_sync(FULL, code, leader);
     const uint32_t peers = __ballot_sync(FULL, code == c);
-    if ((int)(threadIdx.x & 31) == leader) table_add(tv, make_key(site, fmt, (uint32_t)c), __popc(peers), gidx);
+    pend.push(tv, make_key(site, fmt, (uint32_t)c), __popc(peers), gidx);
     pending &= ~peers;
   }
 }

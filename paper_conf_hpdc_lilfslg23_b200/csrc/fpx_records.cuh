@@ -142,30 +142,32 @@ __device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t
 // Exact evaluation + warp aggregation + table update of one record.
 template <int MODE>
 __device__ __forceinline__ void flush_record(const RecDesc& d, const uint32_t* __restrict__ lane_base, int lane,
-                                             uint64_t gidx, const TableView& tv) {
+                                             uint64_t gidx, const TableView& tv, PendingEvents& pend) {
   uint32_t codes, evm;
   const uint32_t cm = eval_record<MODE>(d, lane_base, lane, codes, evm);
   if (MODE == FPX_MODE_DEST) {
-    warp_flush(tv, cm, d.site, fmt_of(d.meta), gidx, [&](int c) {
+    warp_flush(tv, pend, cm, d.site, fmt_of(d.meta), gidx, [&](int c) {
       uint32_t n = 0;
 #pragma unroll
       for (int v = 0; v < 8; ++v) n += (((evm >> v) & 1u) && (((codes >> (4 * v)) & 15u) == (uint32_t)c)) ? 1u : 0u;
       return n;
     });
   } else {
-    warp_flush_single(tv, cm ? (int)codes : CODE_NONE, d.site, fmt_of(d.meta), gidx);
+    warp_flush_single(tv, pend, cm ? (int)codes : CODE_NONE, d.site, fmt_of(d.meta), gidx);
   }
 }
 
 template <int MODE>
 __device__ __noinline__ void exact_tile(const RecDesc* __restrict__ recs, const uint32_t* __restrict__ lane_base,
                                         int lane, uint64_t gidx0, const TableView tv) {
+  PendingEvents pend;
   for (int j = 0; j < TILE; ++j) {
     const RecDesc d = recs[j];
     if (d.mask == 0u) continue;  // warp-uniform
     if (MODE == FPX_MODE_DEST && is_compare(op_of(d.meta))) continue;
-    flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv);
+    flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv, pend);
   }
+  pend.flush(tv);
 }
 
 // Same as exact_tile, reading the tile's k headers from global memory (the
@@ -178,13 +180,15 @@ __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, 
   if ((uint32_t)lane < k) h = hdr_tile[lane];
   const bool ok = (uint32_t)lane < k && record_valid<MODE>(h, arena_planes);
   const uint32_t mask = ok ? h.y : 0u;
+  PendingEvents pend;
   for (uint32_t j = 0; j < k; ++j) {
     const RecDesc d{__shfl_sync(FULL, h.w, j), __shfl_sync(FULL, mask, j), __shfl_sync(FULL, h.z, j),
                     __shfl_sync(FULL, h.x, j)};
     if (d.mask == 0u) continue;  // warp-uniform
     if (MODE == FPX_MODE_DEST && is_compare(op_of(d.meta))) continue;
-    flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv);
+    flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv, pend);
   }
+  pend.flush(tv);
 }
 
 // Plane items of one record for the fast path, by list:

@@ -89,14 +89,16 @@ constexpr int TU = 4;  // vectors per thread per batch
 // Exact per-warp reduction of per-lane kind counts and first offsets.
 __device__ __forceinline__ void flush_kinds(const TableView& tv, uint32_t site, uint32_t fmt, const uint32_t cnt[3],
                                             const uint32_t first_off[3], uint64_t idx0) {
+  PendingEvents pend;
 #pragma unroll
   for (int k = 0; k < 3; ++k) {
     const uint32_t tot = __reduce_add_sync(FULL, cnt[k]);
     if (tot) {
       const uint32_t f = __reduce_min_sync(FULL, first_off[k]);
-      if ((threadIdx.x & 31) == 0) table_add(tv, make_key(site, fmt, (uint32_t)k), tot, idx0 + f);
+      pend.push(tv, make_key(site, fmt, (uint32_t)k), tot, idx0 + f);
     }
   }
+  pend.flush(tv);  // the (at most 3) kinds update the table in parallel
 }
 
 static_assert(TU == 4, "tensor_exact takes four vectors");
