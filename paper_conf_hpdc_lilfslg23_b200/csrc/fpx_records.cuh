@@ -59,7 +59,7 @@ __device__ __forceinline__ uint32_t lane_ext(uint32_t m, int lane) {
 // codes for count_of().
 template <int MODE>
 __device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t* __restrict__ lane_base, int lane,
-                                                uint32_t& codes, uint32_t& evm) {
+                                                uint32_t& codes, uint32_t& evm, const uint32_t* staged = nullptr) {
   codes = 0;
   evm = 0;
   if (((d.mask >> lane) & 1u) == 0u) return 0u;
@@ -70,7 +70,9 @@ __device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t
   uint32_t ns_words = 0;
   if (MODE != FPX_MODE_DEST) ns_words = nsrc * sw;
   else if (have_div) ns_words = 2 * sw;
-  const uint32_t* p = lane_base + (uint64_t)d.val_off * 32;
+  // `staged`: this lane's word of the record's first plane in the shared-memory
+  // stage, which then holds every plane read below (no HBM re-read)
+  const uint32_t* p = staged ? staged : lane_base + (uint64_t)d.val_off * 32;
   uint32_t dv[4], sv[6];
 #pragma unroll
   for (uint32_t k = 0; k < 4; ++k) dv[k] = k < dw ? p[(uint64_t)k * 32] : 0u;
@@ -142,9 +144,10 @@ __device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t
 // Exact evaluation + warp aggregation + table update of one record.
 template <int MODE>
 __device__ __forceinline__ void flush_record(const RecDesc& d, const uint32_t* __restrict__ lane_base, int lane,
-                                             uint64_t gidx, const TableView& tv, PendingEvents& pend) {
+                                             uint64_t gidx, const TableView& tv, PendingEvents& pend,
+                                             const uint32_t* staged = nullptr) {
   uint32_t codes, evm;
-  const uint32_t cm = eval_record<MODE>(d, lane_base, lane, codes, evm);
+  const uint32_t cm = eval_record<MODE>(d, lane_base, lane, codes, evm, staged);
   if (MODE == FPX_MODE_DEST) {
     warp_flush(tv, pend, cm, d.site, fmt_of(d.meta), gidx, [&](int c) {
       uint32_t n = 0;
@@ -170,23 +173,38 @@ __device__ __noinline__ void exact_tile(const RecDesc* __restrict__ recs, const 
   pend.flush(tv);
 }
 
-// Same as exact_tile, reading the tile's k headers from global memory (the
-// record-scan ring keeps no header copy in shared memory).
-template <int MODE>
+// Same as exact_tile for the TMA ring: the tile's k headers are re-read from
+// global memory, while every plane the mode needs is read from the tile's
+// shared-memory stage (`stage_lane` = this lane's word of slot 0; a record's
+// planes sit at the exclusive prefix sum of the needed-plane counts, exactly
+// as the producer laid them out).  `needed(meta)` gives that count for a
+// valid, active record (0 for DIV records, which the producer does not stage:
+// their sources come from global memory).
+template <int MODE, typename Needed>
 __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
-                                            const uint32_t* __restrict__ lane_base, int lane, uint64_t gidx0,
-                                            const TableView tv) {
+                                            const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
+                                            int lane, uint64_t gidx0, const TableView tv, Needed needed) {
   uint4 h = make_uint4(0u, 0u, 0u, 0u);
   if ((uint32_t)lane < k) h = hdr_tile[lane];
   const bool ok = (uint32_t)lane < k && record_valid<MODE>(h, arena_planes);
   const uint32_t mask = ok ? h.y : 0u;
+  const uint32_t c = (ok && mask != 0u) ? needed(h.z) : 0u;
+  uint32_t slot = c;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t t = __shfl_up_sync(FULL, slot, o);
+    if (lane >= o) slot += t;
+  }
+  slot -= c;
+  const uint32_t staged_slot = c != 0u ? slot : 0xFFFFFFFFu;
   PendingEvents pend;
   for (uint32_t j = 0; j < k; ++j) {
     const RecDesc d{__shfl_sync(FULL, h.w, j), __shfl_sync(FULL, mask, j), __shfl_sync(FULL, h.z, j),
                     __shfl_sync(FULL, h.x, j)};
+    const uint32_t sl = __shfl_sync(FULL, staged_slot, j);
     if (d.mask == 0u) continue;  // warp-uniform
     if (MODE == FPX_MODE_DEST && is_compare(op_of(d.meta))) continue;
-    flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv, pend);
+    flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv, pend, sl != 0xFFFFFFFFu ? stage_lane + sl * 32 : nullptr);
   }
   pend.flush(tv);
 }

@@ -406,7 +406,12 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       consume_list<FPX_BF16, true>(w, seg[7], seg[8], ia, pa, g, q);
     }
     if (__any_sync(FULL, w.hit()) || m.force)
-      exact_tile_hdr<MODE>(hdr + (m.gidx0 - base_index), m.k, arena_planes, lane_base, lane, m.gidx0, tv);
+      exact_tile_hdr<MODE>(hdr + (m.gidx0 - base_index), m.k, arena_planes, lane_base, sm.planes[s] + lane, lane,
+                           m.gidx0, tv, [](uint32_t meta) {
+                             bool f;
+                             const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, f, f);
+                             return fmt_of(meta) == FPX_FP64 ? 2u * ni : ni;
+                           });
   }
 }
 
