@@ -231,6 +231,23 @@ fpx_status fpx_scan_records(fpx_handle h, const fpx_rec_hdr* d_hdr, uint64_t n_r
 fpx_status fpx_scan_tensor(fpx_handle h, const void* d_ptr, uint64_t n_elems, uint32_t fmt,
                            uint32_t site, uint64_t base_index, void* stream);
 
+/* Many tensors in ONE launch (e.g. every module output of a forward pass, the
+ * activation detector of SURVEY §8 f1): descs[i] is scanned exactly as
+ * fpx_scan_tensor(h, ptr, n_elems, fmt, site, base_index) would.  descs is
+ * host memory (copied before the call returns); the device pointers must stay
+ * valid until the stream passes the scan.  n == 0 is a no-op.  Errors:
+ * FPX_ERR_INVALID (bad fmt / alignment in any descriptor: nothing is
+ * enqueued), FPX_ERR_NOMEM, FPX_ERR_CUDA. */
+typedef struct {
+  const void* ptr;       /* device pointer, aligned to the element size */
+  uint64_t n_elems;
+  uint64_t base_index;
+  uint32_t fmt;          /* FPX_FP32..FPX_BF16 */
+  uint32_t site;
+} fpx_tensor_desc;       /* 32 bytes */
+
+fpx_status fpx_scan_tensors(fpx_handle h, const fpx_tensor_desc* descs, uint32_t n, void* stream);
+
 /* Synchronise the last scan's stream and copy entries, ascending by key, into
  * caller-allocated host memory.  flags = FPX_FETCH_ALL: every entry;
  * FPX_FETCH_NEW: only keys first inserted since the previous FETCH_NEW call

@@ -33,6 +33,12 @@ struct fpx_ctx {
   void* d_temp = nullptr;
   size_t temp_bytes = 0;
   Ctl* h_ctl = nullptr;  // pinned mirror of the counters
+  // fpx_scan_tensors: device entry table + pinned staging (reused once the
+  // previous copy completed)
+  ListEntry* d_list = nullptr;
+  ListEntry* h_list = nullptr;
+  uint32_t list_cap = 0;
+  cudaEvent_t list_copied = nullptr;
 };
 
 namespace {
@@ -233,6 +239,75 @@ fpx_status fpx_scan_tensor(fpx_handle h, const void* d_ptr, uint64_t n_elems, ui
   if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   CK(launch_scan_tensor(d_ptr, n_elems, fmt, site, base_index, h->tv, h->num_sms, s));
+  h->last_stream = s;
+  return FPX_OK;
+}
+
+fpx_status fpx_scan_tensors(fpx_handle h, const fpx_tensor_desc* descs, uint32_t n, void* stream) {
+  if (!h || (n && !descs)) return FPX_ERR_INVALID;
+  // validate everything before enqueuing anything
+  uint32_t m = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    const fpx_tensor_desc& d = descs[i];
+    if (d.fmt > FPX_BF16) return FPX_ERR_INVALID;
+    if (d.n_elems == 0) continue;
+    const uintptr_t es = d.fmt == FPX_FP64 ? 8 : d.fmt == FPX_FP32 ? 4 : 2;
+    if (!d.ptr || (reinterpret_cast<uintptr_t>(d.ptr) % es) != 0) return FPX_ERR_INVALID;
+    if (d.base_index + d.n_elems < d.base_index) return FPX_ERR_INVALID;
+    ++m;
+  }
+  if (m == 0) return FPX_OK;
+  DeviceGuard g(h->device);
+  if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (!h->list_copied) CK(cudaEventCreateWithFlags(&h->list_copied, cudaEventDisableTiming));
+  CK(cudaEventSynchronize(h->list_copied));  // the staging buffer's previous copy is done
+  if (m > h->list_cap) {
+    if (h->d_list) {
+      CK(cudaStreamSynchronize(h->last_stream));  // earlier launches may still read the old table
+      CK(cudaFree(h->d_list));
+    }
+    if (h->h_list) CK(cudaFreeHost(h->h_list));
+    h->d_list = nullptr;
+    h->h_list = nullptr;
+    uint32_t cap = 64;
+    while (cap < m) cap *= 2;
+    if (cudaMalloc(&h->d_list, sizeof(ListEntry) * cap) != cudaSuccess ||
+        cudaMallocHost(&h->h_list, sizeof(ListEntry) * cap) != cudaSuccess) {
+      cudaGetLastError();
+      h->list_cap = 0;
+      return FPX_ERR_NOMEM;
+    }
+    h->list_cap = cap;
+  }
+  uint64_t vsum = 0, ssum = 0;
+  uint32_t j = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    const fpx_tensor_desc& d = descs[i];
+    if (d.n_elems == 0) continue;
+    const uint32_t es = d.fmt == FPX_FP64 ? 8u : d.fmt == FPX_FP32 ? 4u : 2u;
+    const uint32_t V = 16u / es;
+    const uintptr_t a = reinterpret_cast<uintptr_t>(d.ptr);
+    uint64_t head = ((16u - (uint32_t)(a & 15u)) & 15u) / es;
+    if (head > d.n_elems) head = d.n_elems;
+    const uint64_t nvec = (d.n_elems - head) / V;
+    const uint64_t tail = d.n_elems - head - nvec * V;
+    ListEntry& e = h->h_list[j++];
+    e.ptr = static_cast<const uint8_t*>(d.ptr);
+    e.base = d.base_index;
+    e.vbegin = vsum;
+    e.sbegin = ssum;
+    e.nvec = nvec;
+    e.head = (uint32_t)head;
+    e.tail = (uint32_t)tail;
+    e.fmt = d.fmt;
+    e.site = d.site;
+    vsum += nvec;
+    ssum += head + tail;
+  }
+  CK(cudaMemcpyAsync(h->d_list, h->h_list, sizeof(ListEntry) * m, cudaMemcpyHostToDevice, s));
+  CK(cudaEventRecord(h->list_copied, s));
+  CK(launch_scan_tensor_list(h->d_list, m, vsum, ssum, h->tv, h->num_sms, s));
   h->last_stream = s;
   return FPX_OK;
 }
@@ -463,6 +538,9 @@ fpx_status fpx_close(fpx_handle h) {
       cudaFree(h->tv.ctl);
     }
     cudaFreeHost(h->h_ctl);
+    if (h->h_list) cudaFreeHost(h->h_list);
+    if (h->d_list) cudaFree(h->d_list);
+    if (h->list_copied) cudaEventDestroy(h->list_copied);
     for (void* p : {(void*)h->d_keys, (void*)h->d_counts, (void*)h->d_first, (void*)h->d_keys2, (void*)h->d_idx,
                     (void*)h->d_idx2, (void*)h->d_n, h->d_temp})
       if (p) cudaFree(p);

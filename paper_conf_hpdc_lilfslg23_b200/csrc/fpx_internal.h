@@ -42,6 +42,18 @@ struct TableView {
   Ctl* ctl;
 };
 
+// One tensor of a fused multi-tensor scan (host-prepared, device-resident).
+struct alignas(16) ListEntry {
+  const uint8_t* ptr;   // tensor base
+  uint64_t base;        // first_index of element 0
+  uint64_t vbegin;      // first body vector of this tensor in the launch
+  uint64_t sbegin;      // first head/tail scalar of this tensor in the launch
+  uint64_t nvec;        // 16-B body vectors (starting after `head` elements)
+  uint32_t head, tail;  // scalars before / after the aligned body
+  uint32_t fmt, site;
+};
+static_assert(sizeof(ListEntry) == 64, "list entry is 64 B");
+
 // ---- launchers (fpx_scan_records.cu, fpx_scan_tensor.cu, fpx_table.cu) --------------------------------
 // variant 0 = TMA ring (default), 1 = register-staged LDG (FPX_OPT_SCAN_LDG ablation)
 cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena,
@@ -49,6 +61,8 @@ cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint
                                 const TableView& tv, int num_sms, uint32_t variant, cudaStream_t s);
 cudaError_t launch_scan_tensor(const void* d_ptr, uint64_t n_elems, uint32_t fmt, uint32_t site,
                                uint64_t base_index, const TableView& tv, int num_sms, cudaStream_t s);
+cudaError_t launch_scan_tensor_list(const ListEntry* d_entries, uint32_t n, uint64_t total_vec,
+                                    uint64_t total_scalar, const TableView& tv, int num_sms, cudaStream_t s);
 cudaError_t launch_table_reset(const TableView& tv, uint64_t slots, cudaStream_t s);
 // Clear only the slots recorded in the new-key log (every occupied slot is
 // there unless the log overflowed, in which case the whole table is cleared),

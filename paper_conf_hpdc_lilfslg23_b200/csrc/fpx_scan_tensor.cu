@@ -198,7 +198,149 @@ cudaError_t launch_tensor_t(const void* d_ptr, uint64_t n, uint32_t site, uint64
   return cudaGetLastError();
 }
 
+
+// ---- many tensors in one launch (fpx_scan_tensors) --------------------------
+// Work items: every 16-B body vector of every tensor (prefix vbegin), then
+// every misaligned-head / ragged-tail scalar (prefix sbegin).  A thread finds
+// its tensor by binary search over the (L1-resident) entry table.  Lanes of a
+// warp may belong to different tensors, so the rare exact path groups lanes by
+// tensor before aggregating.
+__device__ __forceinline__ uint32_t find_entry(const ListEntry* __restrict__ e, uint32_t n, uint64_t w, bool scalar) {
+  uint32_t lo = 0, hi = n - 1;  // last entry whose begin <= w
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi + 1) / 2;
+    const uint64_t b = scalar ? e[mid].sbegin : e[mid].vbegin;
+    if (b <= w) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ uint32_t any_cls(uint32_t fmt, uint32_t lo, uint32_t hi) { return cls_val(fmt, lo, hi); }
+
+__device__ __forceinline__ unsigned long long warp_min_u64(unsigned long long v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned long long t = __shfl_xor_sync(FULL, v, o);
+    v = t < v ? t : v;
+  }
+  return v;
+}
+
+// Per-lane (count, first) for each kind -> grouped by tensor -> table.
+__device__ __noinline__ void list_exact_flush(const ListEntry* __restrict__ ents, int ti, const uint32_t cnt[3],
+                                              const unsigned long long first[3], const TableView tv) {
+  PendingEvents pend;
+#pragma unroll
+  for (int k = 0; k < 3; ++k) {
+    const int code = cnt[k] ? ti : -1;
+    uint32_t pending = __ballot_sync(FULL, code >= 0);
+    while (pending) {
+      const int leader = __ffs(pending) - 1;
+      const int t = __shfl_sync(FULL, code, leader);
+      const bool mine = code == t;
+      const uint32_t peers = __ballot_sync(FULL, mine);
+      const uint32_t tot = __reduce_add_sync(FULL, mine ? cnt[k] : 0u);
+      const unsigned long long f = warp_min_u64(mine ? first[k] : ~0ull);
+      const ListEntry& e = ents[t];
+      pend.push(tv, make_key(e.site, e.fmt, (uint32_t)k), tot, f);
+      pending &= ~peers;
+    }
+  }
+  pend.flush(tv);
+}
+
+__global__ void __launch_bounds__(256, 6)
+k_scan_tensor_list(const ListEntry* __restrict__ ents, uint32_t n_ent, uint64_t total_vec, uint64_t total_scalar,
+                   const TableView tv) {
+  const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  // body vectors (loop bound is warp-uniform so the exact path's collectives see the full warp)
+  const uint64_t vtrips = (total_vec + nthr - 1) / nthr;
+  for (uint64_t it = 0; it < vtrips; ++it) {
+    const uint64_t w = it * nthr + tid;
+    int ti = -1;
+    uint32_t fmt = 0;
+    uint4 q = make_uint4(0u, 0u, 0u, 0u);
+    bool hit = false;
+    if (w < total_vec) {
+      ti = (int)find_entry(ents, n_ent, w, false);
+      const ListEntry& e = ents[ti];
+      fmt = e.fmt;
+      const uint32_t es = fmt == FPX_FP64 ? 8u : fmt == FPX_FP32 ? 4u : 2u;
+      q = ld_stream4(e.ptr + (uint64_t)e.head * es + (w - e.vbegin) * 16);
+      uint32_t mn = 0xFFFFFFFFu, mx = 0u;
+      switch (fmt) {
+        case FPX_FP32: vec_witness<FPX_FP32>(q, mn, mx); hit = witness_hit<FPX_FP32>(mn, mx); break;
+        case FPX_FP64: vec_witness<FPX_FP64>(q, mn, mx); hit = witness_hit<FPX_FP64>(mn, mx); break;
+        case FPX_FP16: vec_witness<FPX_FP16>(q, mn, mx); hit = witness_hit<FPX_FP16>(mn, mx); break;
+        default: vec_witness<FPX_BF16>(q, mn, mx); hit = witness_hit<FPX_BF16>(mn, mx); break;
+      }
+    }
+    if (__any_sync(FULL, hit)) {
+      uint32_t cnt[3] = {0, 0, 0};
+      unsigned long long first[3] = {~0ull, ~0ull, ~0ull};
+      if (hit) {
+        const ListEntry& e = ents[ti];
+        const uint32_t V = fmt == FPX_FP64 ? 2u : fmt == FPX_FP32 ? 4u : 8u;
+        const uint64_t e0 = e.base + e.head + (w - e.vbegin) * V;  // global index of the vector's first value
+        const uint32_t wd[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+        for (uint32_t v = 0; v < 8; ++v) {
+          if (v >= V) break;
+          uint32_t lo, hi = 0;
+          if (fmt == FPX_FP64) { lo = wd[(2 * v) & 3]; hi = wd[(2 * v + 1) & 3]; }
+          else if (fmt == FPX_FP32) lo = wd[v & 3];
+          else lo = (wd[(v / 2) & 3] >> (16 * (v & 1))) & 0xFFFFu;
+          const int k = kind_of_cls(any_cls(fmt, lo, hi));
+#pragma unroll
+          for (int kk = 0; kk < 3; ++kk)
+            if (k == kk) { cnt[kk]++; first[kk] = min(first[kk], (unsigned long long)(e0 + v)); }
+        }
+      }
+      list_exact_flush(ents, hit ? ti : -1, cnt, first, tv);
+    }
+  }
+  // misaligned heads and ragged tails, one scalar per thread
+  const uint64_t strips = (total_scalar + nthr - 1) / nthr;
+  for (uint64_t it = 0; it < strips; ++it) {
+    const uint64_t w = it * nthr + tid;
+    int ti = -1;
+    uint32_t cnt[3] = {0, 0, 0};
+    unsigned long long first[3] = {~0ull, ~0ull, ~0ull};
+    if (w < total_scalar) {
+      ti = (int)find_entry(ents, n_ent, w, true);
+      const ListEntry& e = ents[ti];
+      const uint32_t es = e.fmt == FPX_FP64 ? 8u : e.fmt == FPX_FP32 ? 4u : 2u;
+      const uint32_t V = 16u / es;
+      const uint64_t r = w - e.sbegin;
+      const uint64_t el = r < e.head ? r : e.head + e.nvec * V + (r - e.head);
+      const uint8_t* a = e.ptr + el * es;
+      uint32_t lo = 0, hi = 0;
+      if (es == 8) { lo = *(const uint32_t*)a; hi = *(const uint32_t*)(a + 4); }
+      else if (es == 4) lo = *(const uint32_t*)a;
+      else lo = *(const uint16_t*)a;
+      const int k = kind_of_cls(any_cls(e.fmt, lo, hi));
+#pragma unroll
+      for (int kk = 0; kk < 3; ++kk)
+        if (k == kk) { cnt[kk] = 1; first[kk] = e.base + el; }
+    }
+    const bool any = cnt[0] | cnt[1] | cnt[2];
+    if (__any_sync(FULL, any)) list_exact_flush(ents, any ? ti : -1, cnt, first, tv);
+  }
+}
+
 }  // namespace
+
+cudaError_t launch_scan_tensor_list(const ListEntry* d_entries, uint32_t n, uint64_t total_vec, uint64_t total_scalar,
+                                    const TableView& tv, int num_sms, cudaStream_t s) {
+  if (n == 0 || total_vec + total_scalar == 0) return cudaSuccess;
+  uint64_t blocks = (total_vec + 1023) / 1024;
+  const uint64_t cap = (uint64_t)num_sms * 8;
+  if (blocks > cap) blocks = cap;
+  if (blocks == 0) blocks = 1;
+  k_scan_tensor_list<<<(unsigned)blocks, 256, 0, s>>>(d_entries, n, total_vec, total_scalar, tv);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_scan_tensor(const void* d_ptr, uint64_t n, uint32_t fmt, uint32_t site, uint64_t base_index,
                                const TableView& tv, int num_sms, cudaStream_t s) {

@@ -43,6 +43,11 @@ class IpcTable(ctypes.Structure):
                 ("newlog_capacity", ctypes.c_uint32), ("home_device", ctypes.c_int32), ("magic", ctypes.c_uint32)]
 
 
+class TensorDesc(ctypes.Structure):
+    _fields_ = [("ptr", ctypes.c_void_p), ("n_elems", ctypes.c_uint64), ("base_index", ctypes.c_uint64),
+                ("fmt", ctypes.c_uint32), ("site", ctypes.c_uint32)]
+
+
 class Options(ctypes.Structure):
     _fields_ = [("table_log2_slots", ctypes.c_uint32), ("newlog_capacity", ctypes.c_uint32),
                 ("flags", ctypes.c_uint32)]
@@ -59,6 +64,7 @@ _SIGS = {
     "fpx_open": ([ctypes.c_int, ctypes.POINTER(Options), ctypes.POINTER(_vp)], _st),
     "fpx_scan_records": ([_vp, _vp, _u64, _vp, _u64, _u64, _u32, _vp], _st),
     "fpx_scan_tensor": ([_vp, _vp, _u64, _u32, _u32, _u64, _vp], _st),
+    "fpx_scan_tensors": ([_vp, ctypes.POINTER(TensorDesc), _u32, _vp], _st),
     "fpx_table_fetch": ([_vp, _vp, _u64, _P64, _u32], _st),
     "fpx_table_fetch_device": ([_vp, _vp, _vp, _vp, _u64, _P64, _vp], _st),
     "fpx_table_lookup_device": ([_vp, _vp, _u64, _vp, _vp, _vp], _st),
@@ -175,6 +181,18 @@ class Handle:
         n = t.numel() * t.element_size() // es
         check(lib.fpx_scan_tensor(self._h, t.data_ptr(), n, fmt, site, base_index, _stream_ptr(stream)),
               "fpx_scan_tensor")
+
+    def scan_tensors(self, items, stream=None):
+        """One launch for many tensors: items = [(tensor, site, base_index), ...]
+        (fmt from the dtype).  fpx_scan_tensors."""
+        import torch
+
+        fmts = {torch.float32: FP32, torch.float64: FP64, torch.float16: FP16, torch.bfloat16: BF16}
+        arr = (TensorDesc * max(len(items), 1))()
+        for i, (t, site, base) in enumerate(items):
+            assert t.is_contiguous()
+            arr[i] = TensorDesc(t.data_ptr(), t.numel(), base, fmts[t.dtype], site)
+        check(lib.fpx_scan_tensors(self._h, arr, len(items), _stream_ptr(stream)), "fpx_scan_tensors")
 
     def fetch(self, flags: int = FETCH_ALL, capacity: int | None = None) -> np.ndarray:
         """Entries ascending by key.  Sticky device statuses (bad record, table

@@ -40,9 +40,13 @@ class SelectivePolicy:
 
 class ActivationScanner:
     def __init__(self, model: torch.nn.Module, handle: "fpx.Handle | None" = None, leaf_only: bool = True,
-                 device: int | None = None, policy: SelectivePolicy | None = None):
+                 device: int | None = None, policy: SelectivePolicy | None = None, batch: bool = False):
+        """batch=True: collect every output of a forward call and scan them all
+        with ONE fused launch (fpx_scan_tensors) when the call returns."""
         self.model = model
         self.policy = policy
+        self.batch = batch
+        self._queue = []
         dev = torch.cuda.current_device() if device is None else device
         self.handle = handle if handle is not None else fpx.Handle(dev)
         self._own = handle is None
@@ -57,9 +61,15 @@ class ActivationScanner:
             self.names.append(name or "<root>")
             self._hooks.append(mod.register_forward_hook(self._make_hook(site)))
         self._pre = model.register_forward_pre_hook(self._on_call)
+        self._post = model.register_forward_hook(self._on_return) if batch else None
 
     def _on_call(self, module, args):
         self.calls += 1
+
+    def _on_return(self, module, args, out):
+        if self._queue:
+            self.handle.scan_tensors(self._queue)
+            self._queue = []
 
     def _make_hook(self, site: int):
         def hook(module, args, out):
@@ -73,7 +83,11 @@ class ActivationScanner:
             if out.is_cuda and out.dtype in (torch.float32, torch.float64, torch.float16, torch.bfloat16):
                 t = out if out.is_contiguous() else out.contiguous()
                 assert t.numel() < (1 << SEQ_SHIFT)
-                self.handle.scan_tensor(t, site=site, base_index=(len(self.seq) << SEQ_SHIFT))
+                base = len(self.seq) << SEQ_SHIFT
+                if self.batch:
+                    self._queue.append((t, site, base))
+                else:
+                    self.handle.scan_tensor(t, site=site, base_index=base)
                 self.seq.append((self.calls, site))
         elif isinstance(out, (tuple, list)):
             for o in out:
@@ -101,6 +115,8 @@ class ActivationScanner:
         for h in self._hooks:
             h.remove()
         self._pre.remove()
+        if self._post is not None:
+            self._post.remove()
         self._hooks = []
         if self._own:
             self.handle.close()

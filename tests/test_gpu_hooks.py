@@ -7,7 +7,8 @@ pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
 
 
-def test_activation_scanner_finds_first_nan_module():
+@pytest.mark.parametrize("batch", [False, True], ids=["per-output", "one-launch"])
+def test_activation_scanner_finds_first_nan_module(batch):
     from paper_conf_hpdc_lilfslg23_b200.hooks import ActivationScanner
     from paper_conf_hpdc_lilfslg23_b200 import fpx
 
@@ -17,7 +18,7 @@ def test_activation_scanner_finds_first_nan_module():
         torch.nn.Linear(128, 10),
     ).cuda()
     x = torch.randn(32, 64, device="cuda")
-    sc = ActivationScanner(model)
+    sc = ActivationScanner(model, batch=batch)
     model(x)
     assert sc.first_exception() is None  # clean forward
     with torch.no_grad():

@@ -393,3 +393,38 @@ def test_irregular_layouts(fpx, mode):
     ref = oracle_scan(hdr2, arena, 77, mode)
     assert_same(got, ref.entries())
     assert stats.bad_records == ref.bad_records > 0
+
+
+def test_scan_tensors_one_launch(fpx):
+    """fpx_scan_tensors == one fpx_scan_tensor per descriptor == the oracle,
+    over mixed formats, empty / tiny / misaligned / large tensors and a dense
+    NaN tensor."""
+    g = torch.Generator(device=DEV).manual_seed(11)
+    items = []
+    for i, (dt, n, off) in enumerate([(torch.float32, 0, 0), (torch.float16, 1, 0), (torch.bfloat16, 7, 3),
+                                      (torch.float64, 1001, 1), (torch.float32, 100_003, 2), (torch.float16, 65_537, 5),
+                                      (torch.bfloat16, 333_333, 0), (torch.float64, 12_345, 0), (torch.float32, 4096, 0)]):
+        base = torch.randn(n + off, generator=g, device=DEV).to(dt)
+        t = base[off:]
+        if n > 10:
+            t[:: max(1, n // 17)] = float("nan")
+            t[5:: max(1, n // 7)] = float("-inf")
+        if i == 8:
+            t[:] = float("nan")  # dense
+        items.append((t, 100 + i, 1000 * i))
+    with fpx.Handle(0) as h:
+        h.scan_tensors(items)
+        got = h.fetch()
+    with fpx.Handle(0) as h:
+        for t, site, b in items:
+            if t.numel():
+                h.scan_tensor(t, site=site, base_index=b)
+        single = h.fetch()
+    ref = oracle.Table()
+    for t, site, b in items:
+        if t.numel():
+            host = t.contiguous().view({2: torch.int16, 4: torch.int32, 8: torch.int64}[t.element_size()]).cpu().numpy()
+            ref.scan_tensor(host, {torch.float32: FP32, torch.float64: FP64, torch.float16: FP16,
+                                   torch.bfloat16: BF16}[t.dtype], site=site, base_index=b)
+    assert_same(got, ref.entries())
+    assert_same(single, ref.entries())
