@@ -112,10 +112,6 @@ __global__ void k_gather(const uint64_t* idx, uint64_t n, const uint64_t* c_in, 
   }
 }
 
-struct NotEmpty {
-  __device__ bool operator()(const uint64_t k) const { return k != FPX_KEY_EMPTY; }
-};
-
 unsigned grid_for(uint64_t n) {
   uint64_t b = (n + 255) / 256;
   if (b > 148 * 16) b = 148 * 16;
