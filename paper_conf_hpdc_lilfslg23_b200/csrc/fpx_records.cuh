@@ -224,9 +224,8 @@ __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, 
     // skip records of the tile holding no exceptional value at all: every
     // event needs one among the staged planes (DEST: destination, FLOW:
     // destination or sources); unstaged (DIV) records always go through
-    const uint32_t cj = __shfl_sync(FULL, c, j);
-    if (staged != nullptr &&
-        !__any_sync(FULL, ((d.mask >> lane) & 1u) != 0u && staged_any_ev(fmt_of(d.meta), staged, cj)))
+    if (staged != nullptr && !__any_sync(FULL, ((d.mask >> lane) & 1u) &&
+                                                   staged_any_ev(fmt_of(d.meta), staged, __shfl_sync(FULL, c, j))))
       continue;
     flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv, pend, staged);
   }
