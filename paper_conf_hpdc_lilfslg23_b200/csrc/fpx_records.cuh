@@ -173,22 +173,6 @@ __device__ __noinline__ void exact_tile(const RecDesc* __restrict__ recs, const 
   pend.flush(tv);
 }
 
-// Does this lane hold an exceptional value in the record's c staged planes?
-__device__ __forceinline__ bool staged_any_ev(uint32_t fmt, const uint32_t* p, uint32_t c) {
-  bool ev = false;
-  if (fmt == FPX_FP64) {
-    for (uint32_t q = 0; q + 1 < c; q += 2) ev |= cls_fp64(p[q * 32], p[q * 32 + 32]) != CLS_CLEAN;
-  } else {
-    for (uint32_t q = 0; q < c; ++q) {
-      const uint32_t w = p[q * 32];
-      if (fmt == FPX_FP32) ev |= cls_fp32(w) != CLS_CLEAN;
-      else if (fmt == FPX_FP16) ev |= (cls_fp16(w & 0xFFFFu) | cls_fp16(w >> 16)) != CLS_CLEAN;
-      else ev |= (cls_bf16(w & 0xFFFFu) | cls_bf16(w >> 16)) != CLS_CLEAN;
-    }
-  }
-  return ev;
-}
-
 // Same as exact_tile for the TMA ring: the tile's k headers are re-read from
 // global memory, while every plane the mode needs is read from the tile's
 // shared-memory stage (`stage_lane` = this lane's word of slot 0; a record's
@@ -220,14 +204,7 @@ __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, 
     const uint32_t sl = __shfl_sync(FULL, staged_slot, j);
     if (d.mask == 0u) continue;  // warp-uniform
     if (MODE == FPX_MODE_DEST && is_compare(op_of(d.meta))) continue;
-    const uint32_t* staged = sl != 0xFFFFFFFFu ? stage_lane + sl * 32 : nullptr;
-    // skip records of the tile holding no exceptional value at all: every
-    // event needs one among the staged planes (DEST: destination, FLOW:
-    // destination or sources); unstaged (DIV) records always go through
-    if (staged != nullptr && !__any_sync(FULL, ((d.mask >> lane) & 1u) &&
-                                                   staged_any_ev(fmt_of(d.meta), staged, __shfl_sync(FULL, c, j))))
-      continue;
-    flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv, pend, staged);
+    flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv, pend, sl != 0xFFFFFFFFu ? stage_lane + sl * 32 : nullptr);
   }
   pend.flush(tv);
 }
