@@ -41,5 +41,14 @@ for dt in (torch.float32, torch.float64, torch.float16, torch.bfloat16):
         for a in range(4):
             h.scan_tensor(x[a: x.numel() - a], site=a)
         h.fetch()
+# fused multi-tensor scan: mixed formats, ragged heads / tails, an empty tensor
+xs = [torch.randn(n, device=dev).to(dt) for n, dt in
+      ((70_001, torch.float32), (0, torch.float16), (33_333, torch.bfloat16), (12_345, torch.float64))]
+for i, x in enumerate(xs):
+    if x.numel():
+        x[i::501] = float("inf")
+with fpx.Handle(0) as h:
+    h.scan_tensors([(x[1:] if x.numel() > 1 else x, i, i << 20) for i, x in enumerate(xs)])
+    h.fetch()
 torch.cuda.synchronize()
 print("sanitize workload ok")
