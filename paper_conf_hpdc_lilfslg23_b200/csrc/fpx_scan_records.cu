@@ -104,11 +104,12 @@ struct RingCfg {
 constexpr int NLISTS = 8;
 
 struct StageMeta {
-  uint32_t k;                // records in the tile (0 = no tile)
-  uint32_t force;            // tile holds a record that must take the exact path
-  uint64_t gidx0;            // global index of the tile's first record
-  uint32_t seg[NLISTS + 1];  // list l = items [seg[l], seg[l+1])
-  uint32_t pad[3];
+  uint32_t k;      // records in the tile (0 = no tile)
+  uint32_t force;  // tile holds a record that must take the exact path
+  uint64_t gidx0;  // global index of the tile's first record
+  uint32_t tf;     // packed per-format item counts, full-mask lists (byte = format)
+  uint32_t tp;     // same, partial-mask lists
+  uint32_t pad[2];
 };
 
 template <class C>
@@ -118,9 +119,19 @@ struct alignas(128) WarpSmem {  // 128-B multiple: every warp's planes stay 16-B
   StageMeta meta[C::STAGES];
   uint64_t bar[C::STAGES];
 };
+// Header-decode table, one byte per (opclass < 32, fmt, nsrc, dwords):
+// low nibble = fast-path items (0..4), DECODE_FORCE (DIV: exact path) or
+// DECODE_BAD (meta violates the contract of include/fpx.h); high nibble = the
+// record's arena footprint in planes.  Built per CTA from decode_items().
+constexpr int DECODE_ENTRIES = 4096;
+constexpr uint32_t DECODE_FORCE = 5u, DECODE_BAD = 15u;
+__device__ __forceinline__ uint32_t decode_index(uint32_t meta) { return ((meta >> 3) & 0xFE0u) | (meta & 31u); }
+// meta bits outside the table index that a valid record keeps zero
+constexpr uint32_t META_RESERVED = 0xFFFF80E0u;
+
 template <class C>
 constexpr size_t ring_smem() {
-  return sizeof(WarpSmem<C>) * C::WARPS;
+  return sizeof(WarpSmem<C>) * C::WARPS + DECODE_ENTRIES;
 }
 
 // Header decode for the fast path, branch-free: validity (the contract of
@@ -150,6 +161,41 @@ __device__ __forceinline__ uint32_t decode_items(const uint4 h, uint64_t arena_p
 // arena planes a record occupies (destination + all sources)
 __device__ __forceinline__ uint32_t footprint(uint32_t meta) {
   return dwords_of(meta) + (nsrc_of(meta) << (fmt_of(meta) == FPX_FP64 ? 1u : 0u));
+}
+
+template <int MODE>
+__device__ void build_decode_table(uint8_t* lut) {
+  for (uint32_t i = threadIdx.x; i < (uint32_t)DECODE_ENTRIES; i += blockDim.x) {
+    const uint32_t meta = (i & 31u) | ((i >> 5) << 8);
+    bool ok, force;
+    const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, ok, force);
+    const uint32_t code = !ok ? DECODE_BAD : force ? DECODE_FORCE : ni;
+    lut[i] = (uint8_t)((footprint(meta) << 4) | code);
+  }
+}
+
+// Same result as decode_items() from the table: validity, items, force, footprint.
+__device__ __forceinline__ uint32_t decode_fast(const uint8_t* lut, const uint4 h, uint64_t arena_planes,
+                                                bool inrange, bool& ok, bool& force, uint32_t& foot) {
+  const uint32_t e = lut[decode_index(h.z)];
+  const uint32_t code = e & 15u;
+  foot = e >> 4;
+  const bool v = inrange & (h.x != FPX_SITE_INVALID) & ((h.z & META_RESERVED) == 0u) & (code != DECODE_BAD) &
+                 ((uint64_t)h.w + foot <= arena_planes);
+  ok = v;
+  const bool live = v & (h.y != 0u);
+  force = live & (code == DECODE_FORCE);
+  return (live & (code < DECODE_FORCE)) ? code : 0u;
+}
+
+// inclusive warp scan step: v += value of lane - o (lanes >= o)
+template <int O>
+__device__ __forceinline__ void scan_step(uint32_t& v) {
+  asm("{\n\t.reg .u32 t;\n\t.reg .pred p;\n\t"
+      "shfl.sync.up.b32 t|p, %0, %1, 0, -1;\n\t"
+      "@p add.u32 %0, %0, t;\n\t}"
+      : "+r"(v)
+      : "n"(O));
 }
 
 // planes covered by packed item counts (bytes: FP32, FP64 pairs, FP16, BF16;
@@ -189,8 +235,13 @@ struct Witness {
     }
   }
   __device__ __forceinline__ bool hit() const {
-    return mn32 < 0x00FFFFFEu || mx32 >= 0xFF000000u || mn64 < 0x000FFFFFu || mx64 >= 0x7FF00000u ||
-           min(mn16 & 0xFFFFu, mn16 >> 16) < 0x03FFu || max(mx16 & 0xFFFFu, mx16 >> 16) > 0x7BFFu ||
+    return hit_wide() || hit_half();
+  }
+  __device__ __forceinline__ bool hit_wide() const {
+    return mn32 < 0x00FFFFFEu || mx32 >= 0xFF000000u || mn64 < 0x000FFFFFu || mx64 >= 0x7FF00000u;
+  }
+  __device__ __forceinline__ bool hit_half() const {
+    return min(mn16 & 0xFFFFu, mn16 >> 16) < 0x03FFu || max(mx16 & 0xFFFFu, mx16 >> 16) > 0x7BFFu ||
            min(mnb & 0xFFFFu, mnb >> 16) < 0x007Fu || max(mxb & 0xFFFFu, mxb >> 16) > 0x7F7Fu;
   }
 };
@@ -269,9 +320,12 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   WarpSmem<C>& sm = reinterpret_cast<WarpSmem<C>*>(smem_raw)[warp];
+  uint8_t* lut = smem_raw + sizeof(WarpSmem<C>) * C::WARPS;
+  build_decode_table<MODE>(lut);
+  __syncthreads();
   const uint64_t gw = blockIdx.x * (uint64_t)C::WARPS + warp;
   const uint64_t start = gw * recs_per_warp;
-  if (start >= n) return;  // warp-uniform; no block-wide barriers below
+  if (start >= n) return;  // warp-uniform; no block-wide barriers below this line
   const uint64_t end = min(n, start + recs_per_warp);
   const uint32_t* __restrict__ lane_base = arena + lane;
   const uint64_t policy = policy_evict_first();
@@ -299,7 +353,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     }
     const bool inrange = cursor + lane < end;
     bool ok, force;
-    const uint32_t ni = decode_items<MODE>(h, arena_planes, inrange, ok, force);
+    uint32_t foot_all;
+    const uint32_t ni = decode_fast(lut, h, arena_planes, inrange, ok, force, foot_all);
     const uint32_t mask = ok ? h.y : 0u;
     const uint32_t fmt = fmt_of(h.z);
     const bool part = mask != FULL;
@@ -308,11 +363,11 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const uint32_t c8 = ni << (8 * fmt);
     const uint32_t cf = part ? 0u : c8, cp = part ? c8 : 0u;
     uint32_t sf = cf, sp = cp;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t tf = __shfl_up_sync(FULL, sf, o), tp = __shfl_up_sync(FULL, sp, o);
-      if (lane >= o) { sf += tf; sp += tp; }
-    }
+    scan_step<1>(sf), scan_step<1>(sp);
+    scan_step<2>(sf), scan_step<2>(sp);
+    scan_step<4>(sf), scan_step<4>(sp);
+    scan_step<8>(sf), scan_step<8>(sp);
+    scan_step<16>(sf), scan_step<16>(sp);
     const uint32_t incl_planes = planes_of_items(sf) + planes_of_items(sp);
     // the tile = leading records whose planes fit the stage (>= 1 record)
     const uint32_t fits = __ballot_sync(FULL, inrange && incl_planes <= (uint32_t)PLANES);
@@ -341,22 +396,18 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       for (uint32_t j = 0; j < 4; ++j)  // ni <= 4
         if (j < ni) sm.items[s][at + j] = make_uint2(slot + j * step, mask);
     }
-    if (lane <= NLISTS) {  // seg[l] = items of lists < l
-      const uint32_t f = (uint32_t)lane >> 1;
-      const uint32_t lower = f == 0u ? 0u : (f >= 4u ? (tot_f * 0x01010101u) >> 24
-                                                     : ((tot_f << (32 - 8 * f)) * 0x01010101u) >> 24);
-      m.seg[lane] = lower + ((lane & 1) && f < 4u ? ((tf >> (8 * f)) & 0xFFu) : 0u);
-    }
     if (lane == 0) {
       m.k = k;
       m.force = force_any;
       m.gidx0 = base_index + cursor;
+      m.tf = tf;
+      m.tp = tp;
     }
     // runs of arena-adjacent needed planes -> one bulk copy each.  Records
     // with no arena footprint are transparent; a record whose needed planes
     // stop before the end of its footprint (DEST with sources) ends a run.
     const uint32_t a = h.w;
-    const uint32_t foot = in_tile ? footprint(h.z) : 0u;
+    const uint32_t foot = in_tile ? foot_all : 0u;
     const uint32_t rel = __ballot_sync(FULL, foot != 0u);
     const uint32_t below = rel & ((1u << lane) - 1u);
     const int prev = below ? 31 - __clz(below) : -1;
@@ -391,21 +442,28 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 
     // ---- fast path over the staged planes (lane-quad layout) --------------
     const uint32_t ia = smem_u32(sm.items[s]), pa = smem_u32(sm.planes[s]);
+    // list l = items [seg[l], seg[l+1]); lists in order (fmt, full / partial)
+    const uint32_t tf = m.tf, tp = m.tp;
     uint32_t seg[NLISTS + 1];
+    seg[0] = 0u;
 #pragma unroll
-    for (int l = 0; l <= NLISTS; ++l) seg[l] = m.seg[l];
+    for (int f = 0; f < 4; ++f) {
+      seg[2 * f + 1] = seg[2 * f] + ((tf >> (8 * f)) & 0xFFu);
+      seg[2 * f + 2] = seg[2 * f + 1] + ((tp >> (8 * f)) & 0xFFu);
+    }
     Witness w;
     consume_list<FPX_FP32, false>(w, seg[0], seg[1], ia, pa, g, q);
     consume_list<FPX_FP32, true>(w, seg[1], seg[2], ia, pa, g, q);
     consume_list<FPX_FP64, false>(w, seg[2], seg[3], ia, pa, g, q);
     consume_list<FPX_FP64, true>(w, seg[3], seg[4], ia, pa, g, q);
-    if (seg[4] != seg[8]) {
+    const bool halves = ((tf | tp) >> 16) != 0u;
+    if (halves) {
       consume_list<FPX_FP16, false>(w, seg[4], seg[5], ia, pa, g, q);
       consume_list<FPX_FP16, true>(w, seg[5], seg[6], ia, pa, g, q);
       consume_list<FPX_BF16, false>(w, seg[6], seg[7], ia, pa, g, q);
       consume_list<FPX_BF16, true>(w, seg[7], seg[8], ia, pa, g, q);
     }
-    if (__any_sync(FULL, w.hit()) || m.force)
+    if (__any_sync(FULL, w.hit_wide() || (halves && w.hit_half())) || m.force)
       exact_tile_hdr<MODE>(hdr + (m.gidx0 - base_index), m.k, arena_planes, lane_base, sm.planes[s] + lane, lane,
                            m.gidx0, tv, [](uint32_t meta) {
                              bool f;
@@ -417,7 +475,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 
 // Ring configurations compiled in; FPX_RING (environment, tuning only) picks
 // one, default RING_DEFAULT.
-using Ring0 = RingCfg<16, 2, 52>;
+using Ring0 = RingCfg<16, 2, 50>;
 using Ring1 = RingCfg<20, 2, 40>;
 using Ring2 = RingCfg<28, 2, 28>;
 using Ring3 = RingCfg<24, 2, 32>;
