@@ -659,18 +659,17 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
     return cudaGetLastError();
   }
   // Ring geometry, from interleaved A/B runs on B200 (tools/ab_env.sh,
-  // profiles/r1/ab_rings.txt): 20 warps x 2 stages x 40 planes for traces
-  // with several planes per record (C2, C3, C4a); 24 x 2 x 32 when records
-  // carry about one plane (C5-like FP32 traces, estimated from the arena
-  // density).  Warp counts stay multiples of 4 (one share per SM sub-partition).
-  // FPX_RING (environment, tuning only) overrides.
+  // profiles/r1/ab_rings.txt): 20 warps x 2 stages x 40 planes.  Since the
+  // table-driven decode it also matches 24 x 2 x 32 on one-plane FP32 traces
+  // (C5), which it used to lose to; 12-warp rings with 64-plane or 3-deep
+  // stages lose 10-15 %.  FPX_RING (environment, tuning only) overrides.
   static int forced = -2;
   if (forced == -2) {
     const char* e = getenv("FPX_RING");
     forced = e ? atoi(e) : -1;
   }
   int ring = forced;
-  if (ring < 0) ring = (arena_planes * 4 < n * 5) ? 3 : 1;  // < 1.25 planes per record
+  if (ring < 0) ring = 1;
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   switch (ring) {
     case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
