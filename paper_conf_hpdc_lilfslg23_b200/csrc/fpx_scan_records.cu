@@ -659,17 +659,22 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
     return cudaGetLastError();
   }
   // Ring geometry, from interleaved A/B runs on B200 (tools/ab_env.sh,
-  // profiles/r1/ab_rings.txt): 20 warps x 2 stages x 40 planes.  Since the
-  // table-driven decode it also matches 24 x 2 x 32 on one-plane FP32 traces
-  // (C5), which it used to lose to; 12-warp rings with 64-plane or 3-deep
-  // stages lose 10-15 %.  FPX_RING (environment, tuning only) overrides.
+  // profiles/r1/ab_rings.txt): 20 warps x 2 stages x 40 planes by default;
+  // 12-warp rings with 64-plane or 3-deep stages lose 10-15 %.  FPX_RING
+  // (environment, tuning only) overrides.
   static int forced = -2;
   if (forced == -2) {
     const char* e = getenv("FPX_RING");
     forced = e ? atoi(e) : -1;
   }
   int ring = forced;
-  if (ring < 0) ring = 1;
+  // The 24-warp ring for small traces, which are latency-bound: every warp
+  // gets at most one tile up to 24 x 32 records per SM (C1: 30 us instead of
+  // 45 us).  On large one-plane traces the 20-warp ring wins C5 by 2.8 % (the
+  // 24-warp build is capped at 80 registers and spills) and loses the 1 %
+  // NaN storm S2 by 11 % (its exact path wants more warps): the common case
+  // decides.
+  if (ring < 0) ring = n <= (uint64_t)num_sms * 24 * TILE ? 3 : 1;
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   switch (ring) {
     case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
