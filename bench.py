@@ -383,6 +383,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--variant", default="tma", choices=["tma", "ldg"], help="record-scan kernel (ldg = ablation)")
+    ap.add_argument("--no-warp-agg", action="store_true",
+                    help="ablation: per-lane table updates in the exact path (FPX_OPT_NO_WARP_AGG)")
     ap.add_argument("--debug-one-gpu", action="store_true",
                     help="testing only: every rank on cuda:0 with gloo (exercises the N > 1 code paths on one GPU)")
     ap.add_argument("--merge", default="peer", choices=["nccl", "peer"],
@@ -416,7 +418,8 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
 
-    h = fpx.Handle(local, flags=fpx.OPT_SCAN_LDG if args.variant == "ldg" else 0)
+    hflags = (fpx.OPT_SCAN_LDG if args.variant == "ldg" else 0) | (fpx.OPT_NO_WARP_AGG if args.no_warp_agg else 0)
+    h = fpx.Handle(local, flags=hflags)
     stream = torch.cuda.current_stream(dev)
     if cfg.get("kind") == "tensor":
         wl = TensorWorkload(cfg, rank, seed, dev)
@@ -427,7 +430,7 @@ def main():
     shared, merge_note = None, None
     if world > 1 and args.merge == "peer":
         try:
-            shared = fdist.SharedTable(local, flags=fpx.OPT_SCAN_LDG if args.variant == "ldg" else 0)
+            shared = fdist.SharedTable(local, flags=hflags)
             h.close()
             h = shared.handle
         except RuntimeError as ex:  # no peer / IPC access: fall back to the NCCL merge, and say so
@@ -559,6 +562,8 @@ def main():
                                                                          if shared is not None else
                                                                          " + NCCL merge per step")),
             **({"merge_note": merge_note} if merge_note else {}),
+            **({"ablation": "variant=" + args.variant} if args.variant != "tma" else {}),
+            **({"ablation_agg": "no warp aggregation (FPX_OPT_NO_WARP_AGG)"} if args.no_warp_agg else {}),
         },
         "roofline": {
             "bound": "hbm",

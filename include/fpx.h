@@ -183,13 +183,16 @@ typedef struct fpx_ctx* fpx_handle;
 typedef struct {
   uint32_t table_log2_slots;  /* 0 = default 20 (2^20 slots x 32 B = 32 MiB, L2-sized); valid 4..30 */
   uint32_t newlog_capacity;   /* 0 = default (= number of slots) */
-  uint32_t flags;             /* 0, or FPX_OPT_SCAN_LDG */
+  uint32_t flags;             /* 0, or FPX_OPT_* below (ablations) */
 } fpx_options;
 
-/* Option flags.  FPX_OPT_SCAN_LDG selects the register-staged LDG record-scan
- * kernel instead of the default TMA (cp.async.bulk) shared-memory ring; it
- * computes the same table and exists for ablation measurements only. */
-enum { FPX_OPT_SCAN_LDG = 1 };
+/* Option flags, both ablations that compute the same table:
+ * FPX_OPT_SCAN_LDG selects the register-staged LDG record-scan kernel instead
+ * of the default TMA (cp.async.bulk) shared-memory ring.
+ * FPX_OPT_NO_WARP_AGG turns off warp aggregation (Alg2) in the
+ * record scans' exact path: every lane issues its own table updates, one per
+ * distinct code it holds (SURVEY §8(d) stress ablation; record scans only). */
+enum { FPX_OPT_SCAN_LDG = 1, FPX_OPT_NO_WARP_AGG = 2 };
 
 typedef struct {
   uint64_t bad_records;       /* records skipped by validation (sticky, cumulative) */

@@ -167,7 +167,7 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   *out = nullptr;
   fpx_options o{};
   if (opt) o = *opt;
-  if ((o.flags & ~(uint32_t)FPX_OPT_SCAN_LDG) != 0) return FPX_ERR_INVALID;
+  if ((o.flags & ~(uint32_t)(FPX_OPT_SCAN_LDG | FPX_OPT_NO_WARP_AGG)) != 0) return FPX_ERR_INVALID;
   if (o.table_log2_slots == 0) o.table_log2_slots = 20;
   if (o.table_log2_slots < 4 || o.table_log2_slots > 30) return FPX_ERR_INVALID;
   int ndev = 0;
@@ -205,6 +205,7 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   h->tv.newlog_slot = log_slot;
   h->tv.newlog_cap = cap;
   h->tv.ctl = ctl;
+  h->tv.flags = o.flags & FPX_OPT_NO_WARP_AGG;
   CK(launch_table_reset(h->tv, h->slots, nullptr));
   CK(cudaStreamSynchronize(nullptr));
   *out = h;

@@ -40,6 +40,7 @@ struct TableView {
   unsigned int* newlog_slot;     // slot index of each logged key (for the touched-slot reset)
   unsigned long long newlog_cap;
   Ctl* ctl;
+  uint32_t flags;                // FPX_OPT_NO_WARP_AGG (ablation) or 0
 };
 
 // One tensor of a fused multi-tensor scan (host-prepared, device-resident).

@@ -148,6 +148,22 @@ __device__ __forceinline__ void flush_record(const RecDesc& d, const uint32_t* _
                                              const uint32_t* staged = nullptr) {
   uint32_t codes, evm;
   const uint32_t cm = eval_record<MODE>(d, lane_base, lane, codes, evm, staged);
+  if (tv.flags & FPX_OPT_NO_WARP_AGG) {  // ablation: no warp aggregation, every lane updates the table
+    if (MODE != FPX_MODE_DEST) {
+      if (cm) table_add(tv, make_key(d.site, fmt_of(d.meta), codes), 1u, gidx);  // one code per lane
+      return;
+    }
+    uint32_t mine = cm;  // DEST: bit k = kind k among this lane's values
+    while (mine) {
+      const uint32_t c = (uint32_t)(__ffs(mine) - 1);
+      mine &= mine - 1u;
+      uint32_t n = 0u;
+#pragma unroll
+      for (int v = 0; v < 8; ++v) n += (((evm >> v) & 1u) && (((codes >> (4 * v)) & 15u) == c)) ? 1u : 0u;
+      table_add(tv, make_key(d.site, fmt_of(d.meta), c), n, gidx);
+    }
+    return;
+  }
   if (MODE == FPX_MODE_DEST) {
     warp_flush(tv, pend, cm, d.site, fmt_of(d.meta), gidx, [&](int c) {
       uint32_t n = 0;

@@ -29,6 +29,7 @@ MODE_DEST, MODE_FLOW, MODE_FLOW_DETAIL = 0, 1, 2
 DETAIL_CMP = 4
 FETCH_ALL, FETCH_NEW = 0, 1
 OPT_SCAN_LDG = 1
+OPT_NO_WARP_AGG = 2  # ablation: no warp aggregation in the record scans' exact path
 KEY_EMPTY = 0xFFFFFFFFFFFFFFFF
 
 ENTRY_DTYPE = np.dtype(

@@ -146,7 +146,7 @@ def test_synthetic_trace_parity(fpx, name, recipe, mode, n, sites, variant):
         assert table_dict(got) == expected_from_injections(hdr, inj, base, mode)
 
 
-@pytest.mark.parametrize("variant", [0, 1], ids=["tma", "ldg"])
+@pytest.mark.parametrize("variant", [0, 1, 2, 3], ids=["tma", "ldg", "tma-noagg", "ldg-noagg"])
 def test_dense_nan_storm(fpx, variant):
     p = fpxgen.Params(seed=77, n_records=60_000, n_sites=200, recipe=fpxgen.RECIPE_STRESS, dense_nan=1.0)
     hdr, arena = fpxgen.generate_host(p)
@@ -156,6 +156,20 @@ def test_dense_nan_storm(fpx, variant):
     hdr, arena = fpxgen.generate_host(p)
     got, st, _ = gpu_scan(fpx, hdr, arena, base=3, flags=variant)
     assert_same(got, oracle_scan(hdr, arena, 3).entries())
+
+
+@pytest.mark.parametrize("mode", [DEST, FLOW, FLOW_DETAIL], ids=["dest", "flow", "flow_detail"])
+def test_no_warp_agg_ablation_same_table(fpx, mode):
+    """FPX_OPT_NO_WARP_AGG (per-lane table updates) changes the cost, never the table."""
+    recipe = fpxgen.RECIPE_MIX if mode == DEST else fpxgen.RECIPE_FLOW
+    p = fpxgen.Params(seed=31 + mode, n_records=30_011, n_sites=50, recipe=recipe, p_partial=0.3)
+    hdr, arena = fpxgen.generate_host(p)
+    _, w = fpxgen.plan_injections(p, 3000, flow=mode != DEST)
+    fpxgen.apply_host(w, hdr, arena)
+    exp = oracle_scan(hdr, arena, 11, mode).entries()
+    for flags in (fpx.OPT_NO_WARP_AGG, fpx.OPT_NO_WARP_AGG | fpx.OPT_SCAN_LDG):
+        got, st, _ = gpu_scan(fpx, hdr, arena, base=11, mode=mode, flags=flags)
+        assert_same(got, exp)
 
 
 @pytest.mark.parametrize("variant", [0, 1], ids=["tma", "ldg"])
