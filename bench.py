@@ -45,6 +45,9 @@ CONFIGS = {
     "c4b": dict(name="C4b: fpx_scan_tensor over 40 GB of BF16 model activations (2e10 torch.randn values), "
                      "sparse NaN/INF at 1e-7 plus whole-row NaN bursts",
                 kind="tensor", n=20_000_000_000, dtype="bf16", rho=1e-7, sites=1, mode=0, recipe=-1, p_fp64=0.0),
+    "c4b16": dict(name="C4b (FP16): fpx_scan_tensor over 40 GB of FP16 torch.randn activations (2e10 values; "
+                       "natural subnormals at ~4.9e-5), sparse NaN/INF at 1e-7 plus whole-row NaN bursts",
+                  kind="tensor", n=20_000_000_000, dtype="fp16", rho=1e-7, sites=1, mode=0, recipe=-1, p_fp64=0.0),
     "s1": dict(name="S (stress): 1e7 FP32 FFMA records over 200 sites, every active lane NaN (rho = 1)",
                recipe=4, n=10_000_000, sites=200, p_fp64=0.0, mode=0, n_inj=0, dense=1.0),
     "s2": dict(name="S (stress): 1e7 FP32 FFMA records over 200 sites, NaN density 1e-2",
@@ -167,14 +170,51 @@ def cpu_baseline_oracle(cfg, seed, budget_s: float = 12.0):
         t0 = time.perf_counter()
         t.scan_records(hdr, arena, base_index=0, mode=cfg["mode"])
         dt = time.perf_counter() - t0
-        return t.lane_values, dt
+        return t.lane_values, dt, (hdr.nbytes + arena.nbytes) / n
 
-    lv, dt = run(20_000)
+    lv, dt, _ = run(20_000)
     n = int(min(cfg["n"], max(20_000, 20_000 * budget_s / max(dt, 1e-6))))
-    lv, dt = run(n)
-    return {"value": lv / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+    lv, dt, bpr = run(n)
+    return {"value": lv / dt, "unit": UNIT, "cores": 1, "kind": "oracle", "bytes_per_record": bpr,
             "sample": f"first {n} records of the same {cfg['name'].split(':')[0]} trace (same seed), "
                       f"single-threaded C++ oracle, {dt:.1f} s, {lv} lane-values"}
+
+
+def cpu_baseline_oracle_nc(cfg, seed, single, mem_budget=12e9):
+    """SURVEY §8(d) oracle-Nc: nproc processes of the unmodified oracle over
+    contiguous record shards (~12 GB of trace in total), merged on the host.
+    Time = slowest shard's scan + the host merge (generation excluded, as in
+    the single-thread figure, which is kept as `single_core`)."""
+    procs = os.cpu_count() or 1
+    bpr = single["bytes_per_record"]
+    per = int(max(1000, min(cfg["n"] // procs, mem_budget / procs / bpr)))
+    n_inj = 0 if "n_inj" in cfg else max(1, int(round(cfg.get("rho", 1e-6) * per * 32)))
+    tool = os.path.join(ROOT, "tools", "oracle_shard.py")
+    env = dict(os.environ, CUDA_VISIBLE_DEVICES="")
+    ps = [subprocess.Popen([sys.executable, tool, json.dumps(cfg), str(seed), str(i * per), str(per), str(n_inj)],
+                           stdout=subprocess.PIPE, text=True, env=env) for i in range(procs)]
+    res = []
+    for pr in ps:
+        out, _ = pr.communicate(timeout=600)
+        if pr.returncode != 0:
+            raise RuntimeError(f"oracle shard failed (rc {pr.returncode})")
+        d = json.loads(out.strip().splitlines()[-1])
+        res.append((d["lane_values"], d["seconds"], d["entries"]))
+    t0 = time.perf_counter()
+    merged = {}
+    for _, _, ents in res:
+        for site, kind, flow, fmt, detail, count, first in ents:
+            k = (site, kind, flow, fmt, detail)
+            c = merged.get(k)
+            merged[k] = (count, first) if c is None else (c[0] + count, min(c[1], first))
+    dt_merge = time.perf_counter() - t0
+    lv = sum(r[0] for r in res)
+    dt = max(r[1] for r in res) + dt_merge
+    return {"value": lv / dt, "unit": UNIT, "cores": procs, "kind": "oracle",
+            "sample": f"{procs} processes x {per} records (contiguous shards of the same "
+                      f"{cfg['name'].split(':')[0]} trace, same seed), unmodified C++ oracle per process, slowest "
+                      f"shard {max(r[1] for r in res):.2f} s + host merge {dt_merge:.3f} s, {lv} lane-values",
+            "single_core": {"value": single["value"], "cores": 1, "sample": single["sample"]}}
 
 
 def run_reference(args, cfg, seed):
@@ -294,7 +334,11 @@ class RecordsWorkload:
                 "mode": ["dest", "flow"][self.cfg["mode"]], "planted_events": int(len(self.inj))}
 
     def cpu_baseline(self):
-        return cpu_baseline_oracle(self.cfg, self.seed)
+        single = cpu_baseline_oracle(self.cfg, self.seed)
+        if (os.cpu_count() or 1) == 1:
+            single.pop("bytes_per_record")
+            return single
+        return cpu_baseline_oracle_nc(self.cfg, self.seed, single)
 
 
 class TensorWorkload:

@@ -24,6 +24,54 @@ pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
 
 
+def test_c4b_fp16_randn_natural_subnormals():
+    """C4b's FP16 variant: torch.randn FP16 holds natural subnormals (|x| <
+    2^-14, ~4.9e-5 of the values), so the exact path runs in ~5 % of the
+    batches.  4.3e9 elements (> 2^32: 64-bit first indices), ragged tail,
+    planted NaN / INF.  Per-kind counts and first indices against the IEEE
+    definition evaluated by torch on the same buffer (a property at any
+    size), plus 6 windows element by element against the CPU oracle."""
+    from paper_conf_hpdc_lilfslg23_b200 import fpx
+
+    n = (1 << 32) + 12_345
+    g = torch.Generator(device="cuda").manual_seed(0x5EED0000 + 4)
+    x = torch.empty(n, dtype=torch.float16, device="cuda")
+    chunk = 1 << 30
+    for a in range(0, n, chunk):
+        b = min(n, a + chunk)
+        x[a:b] = torch.randn(b - a, generator=g, device="cuda", dtype=torch.float32).to(torch.float16)
+    x[(1 << 32) + 7] = float("nan")
+    x[123_456_789] = float("inf")
+    x[n - 1] = float("-inf")
+    base = 1_000
+    with fpx.Handle(0) as h:
+        h.scan_tensor(x, site=5, base_index=base)
+        got = h.fetch()
+        assert h.last_status == fpx.OK
+    exp = {}
+    for kind, m in ((fpx.NAN, torch.isnan(x)), (fpx.INF, torch.isinf(x)),
+                    (fpx.SUB, (x.abs() < 2.0 ** -14) & (x != 0))):
+        cnt = int(m.sum())
+        if cnt:
+            first = int(torch.nonzero(m)[0, 0])
+            exp[(5, fpx.FP16, 0, kind)] = [cnt, base + first]
+        del m
+    assert table_dict(got) == exp
+    assert exp[(5, fpx.FP16, 0, fpx.SUB)][0] > 100_000
+
+    rng = np.random.default_rng(3)
+    starts = [0, n - 1_000_003] + [int(v) for v in rng.integers(0, n - 1_000_003, 4)]
+    with fpx.Handle(0) as h:
+        for a in starts:
+            w = x[a: a + 1_000_003]
+            ref = oracle.Table()
+            ref.scan_tensor(w.cpu().numpy().view(np.uint16), fmt=fpx.FP16, site=5, base_index=base + a)
+            h.reset()
+            h.scan_tensor(w, site=5, base_index=base + a)
+            got = h.fetch()
+            assert entries_equal(got, ref.entries()), describe_diff(got, ref.entries())
+
+
 def test_c2_full_size_closed_form_and_windows():
     from paper_conf_hpdc_lilfslg23_b200 import fpx
 
