@@ -518,11 +518,15 @@ def main():
         dist.barrier()
     total_ms = t_start.elapsed_time(t_end)
     kern_ms = float(np.mean([a.elapsed_time(b) for a, b in evs]))
+    per_rank = None
     if world > 1:
         tdev = torch.device("cpu") if dist.get_backend() == "gloo" else dev
-        t = torch.tensor([total_ms, kern_ms], dtype=torch.float64, device=tdev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms, kern_ms = float(t[0]), float(t[1])
+        t = torch.zeros(world, 2, dtype=torch.float64, device=tdev)
+        t[rank, 0], t[rank, 1] = total_ms, kern_ms
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)  # each rank fills its own row
+        per_rank = {"step_ms": [round(float(v) / K, 4) for v in t[:, 0]],
+                    "scan_kernel_ms": [round(float(v), 4) for v in t[:, 1]]}
+        total_ms, kern_ms = float(t[:, 0].max()), float(t[:, 1].max())
     ms_per_step = total_ms / K
 
     if shared is None or rank == 0:
@@ -627,6 +631,7 @@ def main():
         "gpu_launches": K * (3 + (8 if (world > 1 and shared is None) else 0)),
         "cpu_baseline": cpu,
         "e2e": e2e,
+        **({"per_rank": per_rank} if per_rank else {}),
     }
     print(json.dumps(line), flush=True)
     if shared is not None:
