@@ -103,30 +103,41 @@ __device__ __forceinline__ void flush_kinds(const TableView& tv, uint32_t site, 
 
 static_assert(TU == 4, "tensor_exact takes four vectors");
 
-// Exact classification of one hit batch (rare): offsets relative to the
-// warp's lowest vector of the batch, reduced per warp.
+// Exact classification of one thread's hit batch (rare), no warp collectives:
+// only vectors whose own witness fires are classified (FP16 randn: ~5 % of
+// batches hold a natural subnormal, ~0.04 % of vectors), and the per-kind
+// (count, first body offset) go to the CTA's shared accumulators.  Every
+// event of one tensor has the same site and format, so the table sees one
+// update per kind per CTA, at the end of the kernel.
 template <uint32_t FMT>
 __device__ __noinline__ void tensor_exact(uint4 q0, uint4 q1, uint4 q2, uint4 q3, uint64_t v0, uint64_t nthr,
-                                          uint64_t nvec, int lane, uint64_t idx_base, uint32_t site,
-                                          const TableView tv) {
+                                          uint64_t nvec, unsigned long long* s_cnt, unsigned long long* s_first) {
   constexpr uint32_t V = TensorTraits<FMT>::V;
   const uint4 q[TU] = {q0, q1, q2, q3};
-  const uint64_t wv0 = v0 - (uint64_t)lane;
-  uint32_t cnt[3] = {0, 0, 0}, fo[3] = {0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu};
+  uint32_t cnt[3] = {0, 0, 0};
+  unsigned long long fo[3] = {~0ull, ~0ull, ~0ull};
 #pragma unroll
   for (int u = 0; u < TU; ++u) {
     const uint64_t v = v0 + (uint64_t)u * nthr;
     if (v >= nvec) continue;
+    uint32_t mn = 0xFFFFFFFFu, mx = 0u;
+    vec_witness<FMT>(q[u], mn, mx);
+    if (!witness_hit<FMT>(mn, mx)) continue;
 #pragma unroll
     for (uint32_t e = 0; e < V; ++e) {
       const int k = kind_of_cls(vec_cls<FMT>(q[u], e));
-      const uint32_t off = (uint32_t)((v - wv0) * V + e);
+      const unsigned long long off = v * V + e;
 #pragma unroll
       for (int kk = 0; kk < 3; ++kk)
         if (k == kk) { cnt[kk]++; fo[kk] = min(fo[kk], off); }
     }
   }
-  flush_kinds(tv, site, FMT, cnt, fo, idx_base + wv0 * V);
+#pragma unroll
+  for (int k = 0; k < 3; ++k)
+    if (cnt[k]) {
+      atomicAdd(&s_cnt[k], (unsigned long long)cnt[k]);
+      atomicMin(&s_first[k], fo[k]);
+    }
 }
 
 template <uint32_t FMT>
@@ -160,7 +171,14 @@ k_scan_tensor(const uint4* __restrict__ body, uint64_t nvec, const uint8_t* __re
     flush_kinds(tv, site, FMT, ct, ft, base_index + idx_tail);
   }
 
-  // body: batches of TU vectors per thread, grid-stride
+  // body: batches of TU vectors per thread, grid-stride; per-thread control
+  // flow only (no collectives), events accumulate per CTA in shared memory
+  __shared__ unsigned long long s_cnt[3], s_first[3];
+  if (threadIdx.x < 3) {
+    s_cnt[threadIdx.x] = 0ull;
+    s_first[threadIdx.x] = ~0ull;
+  }
+  __syncthreads();
   for (uint64_t v0 = tid; v0 < nvec; v0 += nthr * TU) {
     uint4 q[TU];
 #pragma unroll
@@ -171,9 +189,11 @@ k_scan_tensor(const uint4* __restrict__ body, uint64_t nvec, const uint8_t* __re
     uint32_t mn = 0xFFFFFFFFu, mx = 0u;
 #pragma unroll
     for (int u = 0; u < TU; ++u) vec_witness<FMT>(q[u], mn, mx);
-    if (__any_sync(FULL, witness_hit<FMT>(mn, mx)))
-      tensor_exact<FMT>(q[0], q[1], q[2], q[3], v0, nthr, nvec, lane, base_index + idx_body, site, tv);
+    if (witness_hit<FMT>(mn, mx)) tensor_exact<FMT>(q[0], q[1], q[2], q[3], v0, nthr, nvec, s_cnt, s_first);
   }
+  __syncthreads();
+  if (threadIdx.x < 3 && s_cnt[threadIdx.x] != 0ull)
+    table_add(tv, make_key(site, FMT, threadIdx.x), s_cnt[threadIdx.x], base_index + idx_body + s_first[threadIdx.x]);
 }
 
 template <uint32_t FMT>
