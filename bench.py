@@ -227,7 +227,10 @@ def run_reference(args, cfg, seed):
 
     if cfg.get("kind") == "tensor":
         return run_reference_tensor(args, cfg, seed)
-    # each step: a bounded sample of the workload sized to ~0.25 s of oracle time
+    # Each step: every host core runs the unmodified oracle over its own
+    # contiguous shard of the same trace (persistent worker processes,
+    # tools/oracle_shard.py --serve), ~0.25 s of oracle time per shard; the
+    # step time is the slowest shard plus the host merge of the shard tables.
     probe_n = 20_000
     p = fpxgen.Params(seed=seed, n_records=probe_n, n_sites=cfg["sites"], recipe=cfg["recipe"], p_fp64=cfg["p_fp64"])
     hdr, arena = fpxgen.generate_host(p)
@@ -235,29 +238,56 @@ def run_reference(args, cfg, seed):
     t0 = time.perf_counter()
     t.scan_records(hdr, arena, mode=cfg["mode"])
     dt = time.perf_counter() - t0
-    n = int(max(1000, min(cfg["n"], probe_n * 0.25 / max(dt, 1e-6))))
-    p = fpxgen.Params(seed=seed, n_records=n, n_sites=cfg["sites"], recipe=cfg["recipe"], p_fp64=cfg["p_fp64"])
-    hdr, arena = fpxgen.generate_host(p)
-    _, w = fpxgen.plan_injections(p, max(1, int(round(cfg.get("rho", 1e-6) * n * 32))), flow=cfg["mode"] == 1)
-    fpxgen.apply_host(w, hdr, arena)
-    for _ in range(args.warmup):
-        t = oracle.Table()
-        t.scan_records(hdr, arena, mode=cfg["mode"])
-    lv_total, dt_total = 0, 0.0
-    for _ in range(args.steps):
-        t = oracle.Table()
+    procs = os.cpu_count() or 1
+    n = int(max(1000, min(cfg["n"] // procs, probe_n * 0.25 / max(dt, 1e-6))))
+    n_inj = 0 if "n_inj" in cfg else max(1, int(round(cfg.get("rho", 1e-6) * n * 32)))
+    tool = os.path.join(ROOT, "tools", "oracle_shard.py")
+    env = dict(os.environ, CUDA_VISIBLE_DEVICES="")
+    ws = [subprocess.Popen([sys.executable, tool, json.dumps(cfg), str(seed), str(i * n), str(n), str(n_inj),
+                            "--serve"], stdin=subprocess.PIPE, stdout=subprocess.PIPE, text=True, env=env)
+          for i in range(procs)]
+    for w in ws:
+        assert json.loads(w.stdout.readline()).get("ready"), "oracle shard failed to start"
+
+    def step():
+        for w in ws:
+            w.stdin.write("scan\n")
+            w.stdin.flush()
+        res = [json.loads(w.stdout.readline()) for w in ws]
         t0 = time.perf_counter()
-        t.scan_records(hdr, arena, mode=cfg["mode"])
-        dt_total += time.perf_counter() - t0
-        lv_total += t.lane_values
+        merged = {}
+        for r in res:
+            for site, kind, flow, fmt, detail, count, first in r["entries"]:
+                k = (site, kind, flow, fmt, detail)
+                c = merged.get(k)
+                merged[k] = (count, first) if c is None else (c[0] + count, min(c[1], first))
+        return sum(r["lane_values"] for r in res), max(r["seconds"] for r in res) + time.perf_counter() - t0
+
+    try:
+        for _ in range(args.warmup):
+            step()
+        lv_total, dt_total = 0, 0.0
+        for _ in range(args.steps):
+            lv, dt = step()
+            lv_total += lv
+            dt_total += dt
+    finally:
+        for w in ws:
+            try:
+                w.stdin.write("quit\n")
+                w.stdin.close()
+            except OSError:
+                pass
+            w.wait(timeout=60)
     value = lv_total / dt_total
-    sample = f"first {n} records of the {cfg['name'].split(':')[0]} trace per step (same seed), single-threaded oracle"
+    sample = (f"{procs} processes x {n} records per step (contiguous shards of the {cfg['name'].split(':')[0]} "
+              f"trace, same seed), unmodified C++ oracle per process; step = slowest shard + host merge")
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt_total / args.steps,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": cfg["name"], "records_per_step": n, "mode": ["dest", "flow"][cfg["mode"]]},
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "config": {"workload": cfg["name"], "records_per_step": n * procs, "mode": ["dest", "flow"][cfg["mode"]]},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": procs, "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -272,9 +302,10 @@ def run_reference_tensor(args, cfg, seed):
 
     g = torch.Generator().manual_seed(seed)
     n = 1 << 24
-    x = torch.randn(n, generator=g, dtype=torch.float32).to(torch.bfloat16)
+    dt = {"bf16": torch.bfloat16, "fp16": torch.float16, "fp32": torch.float32}[cfg["dtype"]]
+    x = torch.randn(n, generator=g, dtype=torch.float32).to(dt)
     x[torch.randint(0, n, (max(1, int(cfg["rho"] * n)),), generator=g)] = float("nan")
-    host = x.view(torch.int16).numpy()
+    host = x.view(torch_int_view(x)).numpy()
     fmt = {"bf16": 3, "fp16": 2, "fp32": 0}[cfg["dtype"]]
     for _ in range(args.warmup):
         oracle.Table().scan_tensor(host, fmt, site=0)
@@ -285,7 +316,7 @@ def run_reference_tensor(args, cfg, seed):
         t.scan_tensor(host, fmt, site=0)
         dt_total += time.perf_counter() - t0
     value = n * args.steps / dt_total
-    sample = f"{n} BF16 torch.randn values per step (same recipe as C4b), single-threaded oracle"
+    sample = f"{n} {cfg['dtype'].upper()} torch.randn values per step (same recipe as C4b), single-threaded oracle"
     print(json.dumps({
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt_total / args.steps,

@@ -1,9 +1,12 @@
-"""One shard of the multi-core oracle baseline (bench.py cpu_baseline): generate
-records [r0, r0 + n) of a synthetic trace on the host, plant that shard's
-events, time the unmodified CPU oracle over it, print one JSON line.  Runs as
-its own process (no torch, no CUDA).
+"""One shard of the multi-core oracle (bench.py cpu_baseline and the
+--impl reference arm): generate records [r0, r0 + n) of a synthetic trace on
+the host, plant that shard's events, time the unmodified CPU oracle over it,
+print one JSON line.  Runs as its own process (no torch, no CUDA).
 
-    python tools/oracle_shard.py '<cfg json>' SEED R0 N N_INJ
+    python tools/oracle_shard.py '<cfg json>' SEED R0 N N_INJ [--serve]
+
+--serve: generate once, print {"ready": true}, then scan once per "scan" line
+read from stdin (a fresh table each time) until "quit" or EOF.
 """
 import json
 import os
@@ -24,13 +27,24 @@ def main():
     if n_inj:
         _, w = fpxgen.plan_injections(p, n_inj, flow=cfg["mode"] == 1, r0=r0)
         fpxgen.apply_host(w, hdr, arena)
-    t = oracle.Table()
-    t0 = time.perf_counter()
-    t.scan_records(hdr, arena, base_index=r0, mode=cfg["mode"])
-    dt = time.perf_counter() - t0
-    ents = [[int(e[f]) for f in ("site", "kind", "flow", "fmt", "detail", "count", "first_index")]
-            for e in t.entries()]
-    print(json.dumps({"lane_values": int(t.lane_values), "seconds": dt, "entries": ents}))
+
+    def scan():
+        t = oracle.Table()
+        t0 = time.perf_counter()
+        t.scan_records(hdr, arena, base_index=r0, mode=cfg["mode"])
+        dt = time.perf_counter() - t0
+        ents = [[int(e[f]) for f in ("site", "kind", "flow", "fmt", "detail", "count", "first_index")]
+                for e in t.entries()]
+        print(json.dumps({"lane_values": int(t.lane_values), "seconds": dt, "entries": ents}), flush=True)
+
+    if "--serve" not in sys.argv:
+        scan()
+        return
+    print(json.dumps({"ready": True}), flush=True)
+    for line in sys.stdin:
+        if line.strip() != "scan":
+            break
+        scan()
 
 
 if __name__ == "__main__":
