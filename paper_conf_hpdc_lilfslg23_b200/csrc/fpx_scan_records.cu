@@ -10,15 +10,17 @@
 //   produce   lane j decodes + validates header j (prefetched one tile ahead),
 //             a warp scan assigns each record's needed planes (DEST: the
 //             destination words; FLOW: destination + sources) a contiguous
-//             slot range in the stage; runs of records whose planes are
-//             adjacent in the arena become ONE cp.async.bulk (TMA) copy
-//             global -> shared, completing on the stage's mbarrier.  Tiles
-//             are issued STAGES-1 ahead, so memory parallelism is bounded by
-//             shared memory, not registers.
-//   consume   per plane one conflict-free 32-bit LDS per lane; a few integer
-//             ops per value keep min / max witnesses of "subnormal" and
-//             "exponent all ones"; one vote per tile (the common case at 1e-6
-//             density is "nothing exceptional")
+//             slot range in the stage; when the tile's needed planes are
+//             one arena-contiguous range (the common case: one min-reduce and
+//             one vote decide it) lane 0 issues ONE cp.async.bulk (TMA) copy
+//             global -> shared, otherwise one copy per run of adjacent planes;
+//             copies complete on the stage's mbarrier.  Tiles are issued
+//             STAGES-1 ahead, so memory parallelism is bounded by shared
+//             memory, not registers.
+//   consume   lane-quad layout (8 threads per plane, one 128-bit LDS each);
+//             a few integer ops per value keep min / max witnesses of
+//             "subnormal" and "exponent all ones"; one vote per tile (the
+//             common case at 1e-6 density is "nothing exceptional")
 //   exact     hit tiles only: rec::exact_tile (kind rule, flow states, warp
 //             aggregation, table) — fpx_records.cuh
 //
@@ -338,20 +340,23 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   }
   __syncwarp();
 
+  // cursor = global record index of the next tile; rem = records left in
+  // this warp's range (< 2^31, checked at launch: 32-bit lane tests)
   uint64_t cursor = start;
+  uint32_t rem = (uint32_t)(end - start);
   uint4 h = make_uint4(0, 0, 0, 0);
-  if (cursor + lane < end) h = ld_stream4(hdr + cursor + lane);
+  if ((uint32_t)lane < rem) h = ld_stream4(hdr + cursor + lane);
 
   // Build tile `s` from the prefetched headers and issue its copies.
   auto produce = [&](int s) {
     StageMeta& m = sm.meta[s];
-    if (cursor >= end) {
+    if (rem == 0u) {
       __syncwarp();
       if (lane == 0) m.k = 0;
       __syncwarp();
       return;
     }
-    const bool inrange = cursor + lane < end;
+    const bool inrange = (uint32_t)lane < rem;
     bool ok, force;
     uint32_t foot_all;
     const uint32_t ni = decode_fast(lut, h, arena_planes, inrange, ok, force, foot_all);
@@ -369,9 +374,10 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     scan_step<8>(sf), scan_step<8>(sp);
     scan_step<16>(sf), scan_step<16>(sp);
     const uint32_t incl_planes = planes_of_items(sf) + planes_of_items(sp);
-    // the tile = leading records whose planes fit the stage (>= 1 record)
+    // the tile = leading records whose planes fit the stage (>= 1 record);
+    // incl_planes never decreases over the lanes, so `fits` is a lane prefix
     const uint32_t fits = __ballot_sync(FULL, inrange && incl_planes <= (uint32_t)PLANES);
-    const uint32_t k = ~fits == 0u ? 32u : (uint32_t)(__ffs(~fits) - 1);
+    const uint32_t k = (uint32_t)__popc(fits);
     const bool in_tile = (uint32_t)lane < k;
     const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
     if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
@@ -403,29 +409,45 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       m.tf = tf;
       m.tp = tp;
     }
-    // runs of arena-adjacent needed planes -> one bulk copy each.  Records
-    // with no arena footprint are transparent; a record whose needed planes
-    // stop before the end of its footprint (DEST with sources) ends a run.
+    // Copies.  Common case: every in-tile record with an arena footprint
+    // needs all of it and the footprints are arena-adjacent in record order
+    // (records with no footprint are transparent), i.e. arena plane - stage
+    // slot is the same for all of them: ONE bulk copy of the tile.
     const uint32_t a = h.w;
     const uint32_t foot = in_tile ? foot_all : 0u;
-    const uint32_t rel = __ballot_sync(FULL, foot != 0u);
-    const uint32_t below = rel & ((1u << lane) - 1u);
-    const int prev = below ? 31 - __clz(below) : -1;
-    const uint32_t prev_end = __shfl_sync(FULL, (c == foot) ? a + c : 0xFFFFFFFFu, prev < 0 ? 0 : prev);
-    const bool head = c != 0u && (prev < 0 || prev_end != a);
-    const uint32_t heads = __ballot_sync(FULL, head);
-    const uint32_t above = lane == 31 ? 0u : heads & (0xFFFFFFFFu << (lane + 1));  // heads above this lane
-    const uint32_t next = above ? (uint32_t)(__ffs(above) - 1) : 32u;
-    const uint32_t next_slot_raw = __shfl_sync(FULL, slot, next & 31u);
-    const uint32_t run_end = next < k ? next_slot_raw : total;
-    __syncwarp();
-    if (lane == 0) mbar_arrive_expect_tx(&sm.bar[s], total * 128u);
-    __syncwarp();
-    if (head) bulk_g2s(&sm.planes[s][slot * 32], arena + (uint64_t)a * 32, (run_end - slot) * 128u, &sm.bar[s], policy);
+    const uint32_t d = a - slot;
+    const uint32_t dmin = __reduce_min_sync(FULL, foot != 0u ? d : 0xFFFFFFFFu);
+    const bool one_run = __all_sync(FULL, foot == 0u || (c == foot && d == dmin)) &&
+                         (uint64_t)dmin + total <= 0x100000000ull;
+    if (one_run) {
+      if (lane == 0) {
+        mbar_arrive_expect_tx(&sm.bar[s], total * 128u);
+        if (total != 0u) bulk_g2s(&sm.planes[s][0], arena + (uint64_t)dmin * 32, total * 128u, &sm.bar[s], policy);
+      }
+    } else {
+      // general case: runs of arena-adjacent needed planes -> one bulk copy
+      // each.  A record whose needed planes stop before the end of its
+      // footprint (DEST with sources) ends a run.
+      const uint32_t rel = __ballot_sync(FULL, foot != 0u);
+      const uint32_t below = rel & ((1u << lane) - 1u);
+      const int prev = below ? 31 - __clz(below) : -1;
+      const uint32_t prev_end = __shfl_sync(FULL, (c == foot) ? a + c : 0xFFFFFFFFu, prev < 0 ? 0 : prev);
+      const bool head = c != 0u && (prev < 0 || prev_end != a);
+      const uint32_t heads = __ballot_sync(FULL, head);
+      const uint32_t above = lane == 31 ? 0u : heads & (0xFFFFFFFFu << (lane + 1));  // heads above this lane
+      const uint32_t next = above ? (uint32_t)(__ffs(above) - 1) : 32u;
+      const uint32_t next_slot_raw = __shfl_sync(FULL, slot, next & 31u);
+      const uint32_t run_end = next < k ? next_slot_raw : total;
+      if (lane == 0) mbar_arrive_expect_tx(&sm.bar[s], total * 128u);
+      __syncwarp();
+      if (head)
+        bulk_g2s(&sm.planes[s][slot * 32], arena + (uint64_t)a * 32, (run_end - slot) * 128u, &sm.bar[s], policy);
+    }
     // advance and prefetch the next tile's headers
     cursor += k;
+    rem -= k;
     h = make_uint4(0, 0, 0, 0);
-    if (cursor + lane < end) h = ld_stream4(hdr + cursor + lane);
+    if ((uint32_t)lane < rem) h = ld_stream4(hdr + cursor + lane);
   };
 
   uint32_t phase = 0;  // bit s = parity to wait for on stage s
@@ -500,6 +522,7 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
   const uint64_t warps = (uint64_t)num_sms * C::WARPS;
   uint64_t per = (n + warps - 1) / warps;
   per = (per + TILE - 1) / TILE * TILE;
+  if (per >= (1ull << 31)) return cudaErrorInvalidValue;  // the kernel counts a warp's records in 32 bits
   const uint64_t blocks = ((n + per - 1) / per + C::WARPS - 1) / C::WARPS;
   k_scan_records_tma<MODE, C><<<(unsigned)blocks, C::WARPS * 32, ring_smem<C>(), s>>>(hdr, n, arena, arena_planes,
                                                                                       base_index, per, tv);
