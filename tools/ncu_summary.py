@@ -23,6 +23,18 @@ WANT = [
     "lts__t_sectors_srcunit_tex_op_read.sum", "lts__t_sectors_op_atom.sum", "lts__t_sectors_op_red.sum",
     "smsp__thread_inst_executed_per_inst_executed.ratio", "sm__cycles_elapsed.avg.per_second",
     "lts__t_sector_hit_rate.pct", "l1tex__t_sector_hit_rate.pct",
+    # warp divergence (north star: "warp-divergence stats")
+    "smsp__sass_average_branch_targets_threads_uniform.pct", "smsp__branch_targets_threads_divergent",
+    "smsp__inst_executed_op_branch.sum",
+    # L2 atomics / reductions issued by the table stage (north star: "L2 atomic throughput")
+    "lts__t_requests_srcunit_tex_op_atom_dot_cas.sum", "lts__t_requests_srcunit_tex_op_atom_dot_alu.sum",
+    "lts__t_requests_srcunit_tex_op_red.sum", "lts__d_atomic_input_cycles_active.avg.pct_of_peak_sustained_elapsed",
+    # where warps wait, per issued instruction
+    "smsp__average_warps_issue_stalled_wait_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_short_scoreboard_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_math_pipe_throttle_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_branch_resolving_per_issue_active.ratio",
 ]
 for r in rows[2:]:
     name = r[hdr.index("Kernel Name")]
