@@ -208,9 +208,22 @@ __device__ __forceinline__ uint32_t planes_of_items(uint32_t p) {
 
 // Witnesses of one 32-bit word (no false negatives; exact thresholds in hit()):
 //   FP32  a2 = |x| << 1:  subnormal <=> a2 - 2 < 0xFFFFFE;  INF/NaN <=> a2 >= 0xFF000000
-//   FP64  a3 = |hi| | (lo != 0):  subnormal <=> a3 - 1 < 0xFFFFF;  INF/NaN <=> a3 >= 0x7FF00000
-//   FP16 / BF16 per half:  subnormal <=> h - 1 < 0x3FF / 0x7F;  INF/NaN <=> h >= 0x7C00 / 0x7F80
+//   FP64  a3 = 2|hi| + (lo != 0):  subnormal <=> a3 - 1 < 0x1FFFFF;  INF/NaN <=> a3 >= 0xFFE00000
+//   FP16 / BF16 per doubled half h (see half4):  subnormal <=> h - 2 < 0x7FE / 0xFE;
+//                         INF/NaN <=> h >= 0xF800 / 0xFF00
 // Inactive lanes are masked to zero first (zero is clean in every format).
+// min(x, 1) as one VIMNMX (the compiler otherwise emits ISETP + SEL)
+__device__ __forceinline__ uint32_t umin1(uint32_t x) {
+  uint32_t r;
+  asm("min.u32 %0, %1, 1;" : "=r"(r) : "r"(x));
+  return r;
+}
+// x * 2 + y kept on the FMA pipe (IMAD) instead of an ALU IADD3
+__device__ __forceinline__ uint32_t imad2(uint32_t x, uint32_t y) {
+  uint32_t r;
+  asm("mad.lo.u32 %0, %1, 2, %2;" : "=r"(r) : "r"(x), "r"(y));
+  return r;
+}
 struct Witness {
   uint32_t mn32 = 0xFFFFFFFFu, mx32 = 0u, mn64 = 0xFFFFFFFFu, mx64 = 0u;
   uint32_t mn16 = 0xFFFFFFFFu, mx16 = 0u, mnb = 0xFFFFFFFFu, mxb = 0u;
@@ -220,31 +233,37 @@ struct Witness {
     mx32 = max(mx32, a2);
   }
   __device__ __forceinline__ void fp64(uint32_t lo, uint32_t hi) {
-    const uint32_t a3 = (hi & 0x7FFFFFFFu) | min(lo, 1u);
+    const uint32_t a3 = imad2(hi, umin1(lo));  // 2|hi| + (lo != 0): IMAD on the FMA pipe + one VIMNMX
     mn64 = min(mn64, a3 - 1u);
     mx64 = max(mx64, a3);
   }
-  // packed halves: per-halfword DPX min / max (VIADDMNMX.U16x2, VIMNMX.U16x2)
+  // packed halves, doubled (x + x: FMA pipe): each half's exponent moves to
+  // the top of its halfword and the signs drop out (the low half's sign lands
+  // in bit 0 of the high half, below every threshold that matters); then
+  // per-halfword DPX min / max (VIADDMNMX.U16x2, VIMNMX.U16x2)
   template <bool BF>
-  __device__ __forceinline__ void half2(uint32_t x) {
-    x &= 0x7FFF7FFFu;
-    if (BF) {
-      mnb = __viaddmin_u16x2(x, 0xFFFFFFFFu, mnb);  // h - 1 per half (0 -> 0xFFFF)
-      mxb = __vimax3_u16x2(x, x, mxb);
-    } else {
-      mn16 = __viaddmin_u16x2(x, 0xFFFFFFFFu, mn16);
-      mx16 = __vimax3_u16x2(x, x, mx16);
-    }
+  __device__ __forceinline__ void half4(uint4 x) {
+    x = make_uint4(x.x + x.x, x.y + x.y, x.z + x.z, x.w + x.w);
+    uint32_t& mn = BF ? mnb : mn16;
+    uint32_t& mx = BF ? mxb : mx16;
+    mn = __viaddmin_u16x2(x.x, 0xFFFEFFFEu, mn);  // h - 2 per half (0, 1 -> 0xFFFE, 0xFFFF)
+    mn = __viaddmin_u16x2(x.y, 0xFFFEFFFEu, mn);
+    mn = __viaddmin_u16x2(x.z, 0xFFFEFFFEu, mn);
+    mn = __viaddmin_u16x2(x.w, 0xFFFEFFFEu, mn);
+    mx = __vimax3_u16x2(x.x, x.y, mx);
+    mx = __vimax3_u16x2(x.z, x.w, mx);
   }
   __device__ __forceinline__ bool hit() const {
     return hit_wide() || hit_half();
   }
   __device__ __forceinline__ bool hit_wide() const {
-    return mn32 < 0x00FFFFFEu || mx32 >= 0xFF000000u || mn64 < 0x000FFFFFu || mx64 >= 0x7FF00000u;
+    return mn32 < 0x00FFFFFEu || mx32 >= 0xFF000000u || mn64 < 0x001FFFFFu || mx64 >= 0xFFE00000u;
   }
   __device__ __forceinline__ bool hit_half() const {
-    return min(mn16 & 0xFFFFu, mn16 >> 16) < 0x03FFu || max(mx16 & 0xFFFFu, mx16 >> 16) > 0x7BFFu ||
-           min(mnb & 0xFFFFu, mnb >> 16) < 0x007Fu || max(mxb & 0xFFFFu, mxb >> 16) > 0x7F7Fu;
+    // doubled halves h = 2|x| (+ 1 for a high half whose low half is negative):
+    // subnormal <=> 2 <= h <= 2 * max_mantissa + 1; INF/NaN <=> h >= 2 * exponent mask
+    return min(mn16 & 0xFFFFu, mn16 >> 16) < 0x07FEu || max(mx16 & 0xFFFFu, mx16 >> 16) >= 0xF800u ||
+           min(mnb & 0xFFFFu, mnb >> 16) < 0x00FEu || max(mxb & 0xFFFFu, mxb >> 16) >= 0xFF00u;
   }
 };
 
@@ -304,10 +323,7 @@ __device__ __forceinline__ void consume_list(Witness& w, uint32_t b, uint32_t e,
         w.fp32(x.z);
         w.fp32(x.w);
       } else {
-        w.half2<FMT == FPX_BF16>(x.x);
-        w.half2<FMT == FPX_BF16>(x.y);
-        w.half2<FMT == FPX_BF16>(x.z);
-        w.half2<FMT == FPX_BF16>(x.w);
+        w.half4<FMT == FPX_BF16>(x);
       }
     }
   }

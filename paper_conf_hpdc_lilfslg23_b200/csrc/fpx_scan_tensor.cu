@@ -65,12 +65,15 @@ __device__ __forceinline__ void vec_witness(const uint4& q, uint32_t& mn, uint32
       mx = max(mx, a3);
     }
   } else {
-    // packed halves: per-halfword DPX min / max (VIADDMNMX.U16x2, VIMNMX3.U16x2)
-    const uint32_t a = q.x & 0x7FFF7FFFu, b = q.y & 0x7FFF7FFFu, c = q.z & 0x7FFF7FFFu, d = q.w & 0x7FFF7FFFu;
-    mn = __viaddmin_u16x2(a, 0xFFFFFFFFu, mn);  // h - 1 per half (0 -> 0xFFFF)
-    mn = __viaddmin_u16x2(b, 0xFFFFFFFFu, mn);
-    mn = __viaddmin_u16x2(c, 0xFFFFFFFFu, mn);
-    mn = __viaddmin_u16x2(d, 0xFFFFFFFFu, mn);
+    // packed halves, doubled (x + x: FMA pipe): each half's exponent moves to
+    // the top of its halfword and the signs drop out (the low half's sign
+    // lands in bit 0 of the high half, below every threshold that matters);
+    // then per-halfword DPX min / max (VIADDMNMX.U16x2, VIMNMX3.U16x2)
+    const uint32_t a = q.x + q.x, b = q.y + q.y, c = q.z + q.z, d = q.w + q.w;
+    mn = __viaddmin_u16x2(a, 0xFFFEFFFEu, mn);  // h - 2 per half (0, 1 -> 0xFFFE, 0xFFFF)
+    mn = __viaddmin_u16x2(b, 0xFFFEFFFEu, mn);
+    mn = __viaddmin_u16x2(c, 0xFFFEFFFEu, mn);
+    mn = __viaddmin_u16x2(d, 0xFFFEFFFEu, mn);
     mx = __vimax3_u16x2(a, b, mx);
     mx = __vimax3_u16x2(c, d, mx);
   }
@@ -80,8 +83,10 @@ __device__ __forceinline__ bool witness_hit(uint32_t mn, uint32_t mx) {
   if (FMT == FPX_FP32) return mn < 0x00FFFFFEu || mx >= 0xFF000000u;  // subnormal | INF/NaN
   if (FMT == FPX_FP64) return mn < 0x000FFFFFu || mx >= 0x7FF00000u;
   const uint32_t lo = min(mn & 0xFFFFu, mn >> 16), hi = max(mx & 0xFFFFu, mx >> 16);
-  if (FMT == FPX_FP16) return lo < 0x03FFu || hi > 0x7BFFu;
-  return lo < 0x007Fu || hi > 0x7F7Fu;
+  // doubled halves h = 2|x| (+ 1 for a high half with a negative low half):
+  // subnormal <=> 2 <= h <= 2 * max_mantissa + 1; INF/NaN <=> h >= 2 * exponent mask
+  if (FMT == FPX_FP16) return lo < 0x07FEu || hi >= 0xF800u;
+  return lo < 0x00FEu || hi >= 0xFF00u;
 }
 
 constexpr int TU = 4;  // vectors per thread per batch
