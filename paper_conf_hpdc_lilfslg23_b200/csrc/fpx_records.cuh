@@ -54,6 +54,35 @@ __device__ __forceinline__ uint32_t lane_ext(uint32_t m, int lane) {
   return (uint32_t)((int32_t)(m << (31 - lane)) >> 31);
 }
 
+// Destination kinds of one lane of a DEST-mode record: calls f(v, kind) for
+// every destination value v whose Alg1 kind (dest_kind) is an exception.
+// dv = destination words, sv = source words (only read when have_div).
+template <typename F>
+__device__ __forceinline__ void for_each_dest_kind(uint32_t op, uint32_t fmt, uint32_t dw, bool have_div,
+                                                   const uint32_t dv[4], const uint32_t sv[6], F f) {
+  const uint32_t nv = fmt == FPX_FP64 ? dw / 2 : fmt == FPX_FP32 ? dw : 2 * dw;
+#pragma unroll
+  for (uint32_t v = 0; v < 8; ++v) {
+    if (v >= nv) break;
+    uint32_t lo, hi = 0, nlo, nhi = 0, dlo, dhi = 0;  // value, dividend, divisor
+    if (fmt == FPX_FP64) {
+      lo = dv[(2 * v) & 3];
+      hi = dv[(2 * v + 1) & 3];
+      nlo = sv[0]; nhi = sv[1]; dlo = sv[2]; dhi = sv[3];
+    } else if (fmt == FPX_FP32) {
+      lo = dv[v & 3];
+      nlo = sv[0]; dlo = sv[1];
+    } else {
+      const uint32_t sh = 16u * (v & 1u);
+      lo = (dv[(v / 2) & 3] >> sh) & 0xFFFFu;
+      nlo = (sv[0] >> sh) & 0xFFFFu;
+      dlo = (sv[1] >> sh) & 0xFFFFu;
+    }
+    const int k = dest_kind(op, fmt, lo, hi, have_div, nlo, nhi, dlo, dhi);
+    if (k >= 0) f(v, k);
+  }
+}
+
 // Exact evaluation of one record for this lane (both modes).  Returns the
 // bitmask of event codes held by this lane; codes / evm describe per-value
 // codes for count_of().
@@ -80,32 +109,12 @@ __device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t
   for (uint32_t k = 0; k < 6; ++k) sv[k] = k < ns_words ? p[(uint64_t)(dw + k) * 32] : 0u;
 
   if (MODE == FPX_MODE_DEST) {
-    const uint32_t nv = fmt == FPX_FP64 ? dw / 2 : fmt == FPX_FP32 ? dw : 2 * dw;
     uint32_t cm = 0;
-#pragma unroll
-    for (uint32_t v = 0; v < 8; ++v) {
-      if (v >= nv) break;
-      uint32_t lo, hi = 0, nlo, nhi = 0, dlo, dhi = 0;  // value, dividend, divisor
-      if (fmt == FPX_FP64) {
-        lo = dv[(2 * v) & 3];
-        hi = dv[(2 * v + 1) & 3];
-        nlo = sv[0]; nhi = sv[1]; dlo = sv[2]; dhi = sv[3];
-      } else if (fmt == FPX_FP32) {
-        lo = dv[v & 3];
-        nlo = sv[0]; dlo = sv[1];
-      } else {
-        const uint32_t sh = 16u * (v & 1u);
-        lo = (dv[(v / 2) & 3] >> sh) & 0xFFFFu;
-        nlo = (sv[0] >> sh) & 0xFFFFu;
-        dlo = (sv[1] >> sh) & 0xFFFFu;
-      }
-      const int k = dest_kind(op, fmt, lo, hi, have_div, nlo, nhi, dlo, dhi);
-      if (k >= 0) {
-        codes |= (uint32_t)k << (4 * v);
-        evm |= 1u << v;
-        cm |= 1u << k;
-      }
-    }
+    for_each_dest_kind(op, fmt, dw, have_div, dv, sv, [&](uint32_t v, int k) {
+      codes |= (uint32_t)k << (4 * v);
+      evm |= 1u << v;
+      cm |= 1u << k;
+    });
     return cm;
   } else {
     // Analyzer: S = most severe class among the pre-execution sources; src =
@@ -197,7 +206,7 @@ __device__ __noinline__ void exact_tile(const RecDesc* __restrict__ recs, const 
 // valid, active record (0 for DIV records, which the producer does not stage:
 // their sources come from global memory).
 template <int MODE, typename Needed>
-__device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
+__device__ __forceinline__ void exact_tile_records(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
                                             const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
                                             int lane, uint64_t gidx0, const TableView tv, Needed needed) {
   uint4 h = make_uint4(0u, 0u, 0u, 0u);
@@ -223,6 +232,85 @@ __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, 
     flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv, pend, sl != 0xFFFFFFFFu ? stage_lane + sl * 32 : nullptr);
   }
   pend.flush(tv);
+}
+
+// DEST-mode exact path of a TMA tile, transposed: lane j evaluates ALL lanes of
+// record j (the k <= 32 records at once) instead of the warp walking the
+// records one by one; then records with equal keys are combined across the
+// warp (Alg2's warp reduction, over records instead of lanes:
+// __match_any_sync + REDUX) and every group leader updates the table, all in
+// parallel.  Same table as exact_tile_records: count = lane-values per key,
+// first = the smallest record index of the group (lanes are in record order).
+// Shared-memory reads are skewed (lane j reads instrumented lane (t + j) mod
+// 32 at step t) so the 32 lanes hit 32 different banks.  `h`, `c`, `slot`:
+// this lane's header, staged planes and stage slot.
+__device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t mask, uint32_t c, uint32_t slot,
+                                                      const uint32_t* __restrict__ arena, const uint32_t* stage,
+                                                      int lane, uint64_t gidx0, const TableView& tv) {
+  const uint32_t op = op_of(h.z), fmt = fmt_of(h.z), nsrc = nsrc_of(h.z), dw = dwords_of(h.z);
+  const uint32_t sw = sw_of(fmt);
+  const bool have_div = (op == FPX_OP_DIV) && nsrc >= 2 && dw == sw;
+  const uint32_t ns_words = have_div ? 2 * sw : 0u;
+  // per-kind lane-value counts of this record, 16 bits each (<= 32 lanes x 8 values)
+  unsigned long long cnt = 0ull;
+  if (mask != 0u && dw != 0u && !is_compare(op)) {
+    // plane 0 of the record: staged (c != 0) or in global memory (DIV records)
+    const uint32_t* p = c != 0u ? stage + slot * 32 : arena + (uint64_t)h.w * 32;
+    for (uint32_t t = 0; t < 32; ++t) {
+      const uint32_t i = (t + (uint32_t)lane) & 31u;
+      if (((mask >> i) & 1u) == 0u) continue;
+      uint32_t dv[4], sv[6];
+#pragma unroll
+      for (uint32_t w = 0; w < 4; ++w) dv[w] = w < dw ? p[w * 32 + i] : 0u;
+#pragma unroll
+      for (uint32_t w = 0; w < 6; ++w) sv[w] = w < ns_words ? p[(dw + w) * 32 + i] : 0u;
+      for_each_dest_kind(op, fmt, dw, have_div, dv, sv, [&](uint32_t, int kd) { cnt += 1ull << (16 * kd); });
+    }
+  }
+  uint32_t present = 0u;
+#pragma unroll
+  for (int kd = 0; kd < 4; ++kd) present |= ((cnt >> (16 * kd)) & 0xFFFFu) ? 1u << kd : 0u;
+  uint32_t all = __reduce_or_sync(FULL, present);
+  while (all) {
+    const uint32_t kd = (uint32_t)(__ffs(all) - 1);
+    all &= all - 1u;
+    const bool has = (present >> kd) & 1u;
+    // lanes without this kind get lane-unique keys no record can have
+    const unsigned long long key = has ? make_key(h.x, fmt, kd) : FPX_KEY_EMPTY - (unsigned long long)lane;
+    const uint32_t peers = __match_any_sync(FULL, key);
+    if (has) {
+      const uint32_t sum = __reduce_add_sync(peers, (uint32_t)((cnt >> (16 * kd)) & 0xFFFFu));
+      if ((uint32_t)lane == (uint32_t)(__ffs(peers) - 1)) table_add(tv, key, sum, gidx0 + (uint64_t)lane);
+    }
+  }
+}
+
+// Exact path of a hit TMA tile.  DEST mode with one format in the tile goes
+// transposed (exact_tile_transposed); tiles mixing formats (whose lanes would
+// serialise per-format code paths), the analyzer modes and the
+// no-aggregation ablation go record by record (exact_tile_records).
+template <int MODE, typename Needed>
+__device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
+                                            const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
+                                            int lane, uint64_t gidx0, const TableView tv, Needed needed) {
+  if (MODE == FPX_MODE_DEST && !(tv.flags & FPX_OPT_NO_WARP_AGG)) {
+    uint4 h = make_uint4(0u, 0u, 0u, 0u);
+    if ((uint32_t)lane < k) h = hdr_tile[lane];
+    if (__popc(__reduce_or_sync(FULL, (uint32_t)lane < k ? 1u << fmt_of(h.z) : 0u)) == 1) {
+      const bool ok = (uint32_t)lane < k && record_valid<MODE>(h, arena_planes);
+      const uint32_t mask = ok ? h.y : 0u;
+      const uint32_t c = (ok && mask != 0u) ? needed(h.z) : 0u;
+      uint32_t slot = c;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t t = __shfl_up_sync(FULL, slot, o);
+        if (lane >= o) slot += t;
+      }
+      exact_tile_transposed(h, mask, c, slot - c, lane_base - lane, stage_lane - lane, lane, gidx0, tv);
+      return;
+    }
+  }
+  exact_tile_records<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, needed);
 }
 
 // Plane items of one record for the fast path, by list:
