@@ -243,28 +243,82 @@ __device__ __forceinline__ void exact_tile_records(const uint4* __restrict__ hdr
 // first = the smallest record index of the group (lanes are in record order).
 // Shared-memory reads are skewed (lane j reads instrumented lane (t + j) mod
 // 32 at step t) so the 32 lanes hit 32 different banks.  `h`, `c`, `slot`:
-// this lane's header, staged planes and stage slot.
+// this lane's header, staged planes and stage slot; `tile_fmt` the tile's one
+// format.
 __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t mask, uint32_t c, uint32_t slot,
-                                                      const uint32_t* __restrict__ arena, const uint32_t* stage,
-                                                      int lane, uint64_t gidx0, const TableView& tv) {
+                                                      uint32_t tile_fmt, const uint32_t* __restrict__ arena,
+                                                      const uint32_t* stage, int lane, uint64_t gidx0,
+                                                      const TableView& tv) {
   const uint32_t op = op_of(h.z), fmt = fmt_of(h.z), nsrc = nsrc_of(h.z), dw = dwords_of(h.z);
   const uint32_t sw = sw_of(fmt);
   const bool have_div = (op == FPX_OP_DIV) && nsrc >= 2 && dw == sw;
-  const uint32_t ns_words = have_div ? 2 * sw : 0u;
   // per-kind lane-value counts of this record, 16 bits each (<= 32 lanes x 8 values)
   unsigned long long cnt = 0ull;
   if (mask != 0u && dw != 0u && !is_compare(op)) {
     // plane 0 of the record: staged (c != 0) or in global memory (DIV records)
     const uint32_t* p = c != 0u ? stage + slot * 32 : arena + (uint64_t)h.w * 32;
-    for (uint32_t t = 0; t < 32; ++t) {
-      const uint32_t i = (t + (uint32_t)lane) & 31u;
-      if (((mask >> i) & 1u) == 0u) continue;
-      uint32_t dv[4], sv[6];
+    if (have_div) {
+      // a recorded division with its operands (R1): the full per-value rule
+      const uint32_t ns_words = 2 * sw;
+      for (uint32_t t = 0; t < 32; ++t) {
+        const uint32_t i = (t + (uint32_t)lane) & 31u;
+        if (((mask >> i) & 1u) == 0u) continue;
+        uint32_t dv[4], sv[6];
 #pragma unroll
-      for (uint32_t w = 0; w < 4; ++w) dv[w] = w < dw ? p[w * 32 + i] : 0u;
+        for (uint32_t w = 0; w < 4; ++w) dv[w] = w < dw ? p[w * 32 + i] : 0u;
 #pragma unroll
-      for (uint32_t w = 0; w < 6; ++w) sv[w] = w < ns_words ? p[(dw + w) * 32 + i] : 0u;
-      for_each_dest_kind(op, fmt, dw, have_div, dv, sv, [&](uint32_t, int kd) { cnt += 1ull << (16 * kd); });
+        for (uint32_t w = 0; w < 6; ++w) sv[w] = w < ns_words ? p[(dw + w) * 32 + i] : 0u;
+        for_each_dest_kind(op, fmt, dw, have_div, dv, sv, [&](uint32_t, int kd) { cnt += 1ull << (16 * kd); });
+      }
+    } else {
+      // Every other opclass maps the destination CLASS to a kind per record
+      // (dest_kind: RCP -> DIV0 for NaN / INF, nothing for SUB; else the
+      // class), so the loop only counts classes, in the tile's one format
+      // (warp-uniform switch).  Inactive lanes are masked to 0 (clean).
+      uint32_t n_nan = 0u, n_inf = 0u, n_sub = 0u;
+      switch (tile_fmt) {
+        case FPX_FP32:
+          for (uint32_t t = 0; t < 32; ++t) {
+            const uint32_t i = (t + (uint32_t)lane) & 31u, act = 0u - ((mask >> i) & 1u);
+            for (uint32_t w = 0; w < dw; ++w) {
+              const uint32_t a = p[w * 32 + i] & act & 0x7FFFFFFFu;
+              n_nan += a > 0x7F800000u;
+              n_inf += a == 0x7F800000u;
+              n_sub += (a - 1u) < 0x007FFFFFu;
+            }
+          }
+          break;
+        case FPX_FP64:
+          for (uint32_t t = 0; t < 32; ++t) {
+            const uint32_t i = (t + (uint32_t)lane) & 31u, act = 0u - ((mask >> i) & 1u);
+            for (uint32_t w = 0; w < dw; w += 2) {
+              const uint32_t lo = p[w * 32 + i] & act, ah = p[(w + 1) * 32 + i] & act & 0x7FFFFFFFu;
+              const bool mant_nz = ((ah & 0x000FFFFFu) | lo) != 0u, exp_max = ah >= 0x7FF00000u;
+              n_nan += exp_max && mant_nz;
+              n_inf += exp_max && !mant_nz;
+              n_sub += ah < 0x00100000u && mant_nz;
+            }
+          }
+          break;
+        default: {
+          const uint32_t em = tile_fmt == FPX_FP16 ? 0x7C00u : 0x7F80u, mm = tile_fmt == FPX_FP16 ? 0x03FFu : 0x007Fu;
+          for (uint32_t t = 0; t < 32; ++t) {
+            const uint32_t i = (t + (uint32_t)lane) & 31u, act = 0u - ((mask >> i) & 1u);
+            for (uint32_t w = 0; w < dw; ++w) {
+              const uint32_t x = p[w * 32 + i] & act & 0x7FFF7FFFu;
+              const uint32_t lo = x & 0xFFFFu, hi = x >> 16;
+              n_nan += (lo > em) + (hi > em);
+              n_inf += (lo == em) + (hi == em);
+              n_sub += ((lo - 1u) < mm) + ((hi - 1u) < mm);
+            }
+          }
+        }
+      }
+      if (op == FPX_OP_MUFU_RCP || op == FPX_OP_MUFU_RCP64H)
+        cnt = (unsigned long long)(n_nan + n_inf) << (16 * FPX_DIV0);
+      else
+        cnt = (unsigned long long)n_nan << (16 * FPX_NAN) | (unsigned long long)n_inf << (16 * FPX_INF) |
+              (unsigned long long)n_sub << (16 * FPX_SUB);
     }
   }
   uint32_t present = 0u;
@@ -296,7 +350,8 @@ __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, 
   if (MODE == FPX_MODE_DEST && !(tv.flags & FPX_OPT_NO_WARP_AGG)) {
     uint4 h = make_uint4(0u, 0u, 0u, 0u);
     if ((uint32_t)lane < k) h = hdr_tile[lane];
-    if (__popc(__reduce_or_sync(FULL, (uint32_t)lane < k ? 1u << fmt_of(h.z) : 0u)) == 1) {
+    const uint32_t fmts = __reduce_or_sync(FULL, (uint32_t)lane < k ? 1u << fmt_of(h.z) : 0u);
+    if (__popc(fmts) == 1) {
       const bool ok = (uint32_t)lane < k && record_valid<MODE>(h, arena_planes);
       const uint32_t mask = ok ? h.y : 0u;
       const uint32_t c = (ok && mask != 0u) ? needed(h.z) : 0u;
@@ -306,7 +361,8 @@ __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, 
         const uint32_t t = __shfl_up_sync(FULL, slot, o);
         if (lane >= o) slot += t;
       }
-      exact_tile_transposed(h, mask, c, slot - c, lane_base - lane, stage_lane - lane, lane, gidx0, tv);
+      exact_tile_transposed(h, mask, c, slot - c, (uint32_t)(__ffs(fmts) - 1), lane_base - lane, stage_lane - lane,
+                            lane, gidx0, tv);
       return;
     }
   }
