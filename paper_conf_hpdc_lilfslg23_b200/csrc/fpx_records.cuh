@@ -243,12 +243,10 @@ __device__ __forceinline__ void exact_tile_records(const uint4* __restrict__ hdr
 // first = the smallest record index of the group (lanes are in record order).
 // Shared-memory reads are skewed (lane j reads instrumented lane (t + j) mod
 // 32 at step t) so the 32 lanes hit 32 different banks.  `h`, `c`, `slot`:
-// this lane's header, staged planes and stage slot; `tile_fmt` the tile's one
-// format.
+// this lane's header, staged planes and stage slot.
 __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t mask, uint32_t c, uint32_t slot,
-                                                      uint32_t tile_fmt, const uint32_t* __restrict__ arena,
-                                                      const uint32_t* stage, int lane, uint64_t gidx0,
-                                                      const TableView& tv) {
+                                                      const uint32_t* __restrict__ arena, const uint32_t* stage,
+                                                      int lane, uint64_t gidx0, const TableView& tv) {
   const uint32_t op = op_of(h.z), fmt = fmt_of(h.z), nsrc = nsrc_of(h.z), dw = dwords_of(h.z);
   const uint32_t sw = sw_of(fmt);
   const bool have_div = (op == FPX_OP_DIV) && nsrc >= 2 && dw == sw;
@@ -273,10 +271,10 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
     } else {
       // Every other opclass maps the destination CLASS to a kind per record
       // (dest_kind: RCP -> DIV0 for NaN / INF, nothing for SUB; else the
-      // class), so the loop only counts classes, in the tile's one format
-      // (warp-uniform switch).  Inactive lanes are masked to 0 (clean).
+      // class), so the loop only counts classes, per format (lanes of one
+      // format run together).  Inactive lanes are masked to 0 (clean).
       uint32_t n_nan = 0u, n_inf = 0u, n_sub = 0u;
-      switch (tile_fmt) {
+      switch (fmt) {
         case FPX_FP32:
           for (uint32_t t = 0; t < 32; ++t) {
             const uint32_t i = (t + (uint32_t)lane) & 31u, act = 0u - ((mask >> i) & 1u);
@@ -301,7 +299,7 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
           }
           break;
         default: {
-          const uint32_t em = tile_fmt == FPX_FP16 ? 0x7C00u : 0x7F80u, mm = tile_fmt == FPX_FP16 ? 0x03FFu : 0x007Fu;
+          const uint32_t em = fmt == FPX_FP16 ? 0x7C00u : 0x7F80u, mm = fmt == FPX_FP16 ? 0x03FFu : 0x007Fu;
           for (uint32_t t = 0; t < 32; ++t) {
             const uint32_t i = (t + (uint32_t)lane) & 31u, act = 0u - ((mask >> i) & 1u);
             for (uint32_t w = 0; w < dw; ++w) {
@@ -339,10 +337,11 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
   }
 }
 
-// Exact path of a hit TMA tile.  DEST mode with one format in the tile goes
-// transposed (exact_tile_transposed); tiles mixing formats (whose lanes would
-// serialise per-format code paths), the analyzer modes and the
-// no-aggregation ablation go record by record (exact_tile_records).
+// Exact path of a hit TMA tile: DEST mode goes transposed
+// (exact_tile_transposed; a tile mixing formats runs each present format's
+// class loop in turn, still far cheaper than walking the records), the
+// analyzer modes and the no-aggregation ablation record by record
+// (exact_tile_records).  A/B in profiles/r1/ab_producer.txt (ab9-ab16).
 template <int MODE, typename Needed>
 __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
                                             const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
@@ -350,21 +349,17 @@ __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, 
   if (MODE == FPX_MODE_DEST && !(tv.flags & FPX_OPT_NO_WARP_AGG)) {
     uint4 h = make_uint4(0u, 0u, 0u, 0u);
     if ((uint32_t)lane < k) h = hdr_tile[lane];
-    const uint32_t fmts = __reduce_or_sync(FULL, (uint32_t)lane < k ? 1u << fmt_of(h.z) : 0u);
-    if (__popc(fmts) == 1) {
-      const bool ok = (uint32_t)lane < k && record_valid<MODE>(h, arena_planes);
-      const uint32_t mask = ok ? h.y : 0u;
-      const uint32_t c = (ok && mask != 0u) ? needed(h.z) : 0u;
-      uint32_t slot = c;
+    const bool ok = (uint32_t)lane < k && record_valid<MODE>(h, arena_planes);
+    const uint32_t mask = ok ? h.y : 0u;
+    const uint32_t c = (ok && mask != 0u) ? needed(h.z) : 0u;
+    uint32_t slot = c;
 #pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t t = __shfl_up_sync(FULL, slot, o);
-        if (lane >= o) slot += t;
-      }
-      exact_tile_transposed(h, mask, c, slot - c, (uint32_t)(__ffs(fmts) - 1), lane_base - lane, stage_lane - lane,
-                            lane, gidx0, tv);
-      return;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(FULL, slot, o);
+      if (lane >= o) slot += t;
     }
+    exact_tile_transposed(h, mask, c, slot - c, lane_base - lane, stage_lane - lane, lane, gidx0, tv);
+    return;
   }
   exact_tile_records<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, needed);
 }
