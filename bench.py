@@ -57,6 +57,21 @@ CONFIGS = {
 }
 
 
+# The paper's headline (context, not the target: another metric on other hardware).
+PAPER_CONTEXT = {
+    "claim": "GPU-FPX vs BinFPE: 16x geomean end-to-end runtime speedup of NVBit-instrumented programs",
+    "hardware": "RTX 2070 SUPER (Turing) + Ryzen 5 3600, or RTX 3060 (Ampere) + i9-10900K",
+    "workload": "151 HPC / ML programs, FP32 + FP64 SASS",
+    "cite": "PAPER.md:29 (abstract), PAPER.md:462 (machines); BASELINE.md",
+    "comparable": False,
+}
+
+
+def config_seed(name: str) -> int:
+    """The seed of a config's synthetic input (0x5EED0000 + config)."""
+    return 0x5EED0000 + list(CONFIGS).index(name) + 1
+
+
 def load_peak():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -469,7 +484,7 @@ def main():
     cfg = dict(CONFIGS[args.config])
     if args.records:
         cfg["n"] = args.records
-    seed = 0x5EED0000 + list(CONFIGS).index(args.config) + 1
+    seed = config_seed(args.config)
 
     if args.impl == "reference":
         return run_reference(args, cfg, seed)
@@ -663,6 +678,7 @@ def main():
         "cpu_baseline": cpu,
         "e2e": e2e,
         **({"per_rank": per_rank} if per_rank else {}),
+        "paper_context": PAPER_CONTEXT,
     }
     print(json.dumps(line), flush=True)
     if shared is not None:
