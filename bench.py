@@ -30,6 +30,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "lane-values classified/sec"
+L2_BYTES = 126 << 20  # B200 L2
 UNIT = "lane-values/s"
 
 # Workloads (BASELINE.json configs); C2 is the headline.
@@ -551,18 +552,30 @@ def main():
     K = args.steps
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
     t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    # Inputs that fit the 126 MB L2 (C1) would be re-read from L2 by every
+    # step: write a 2 x L2 buffer between steps instead, outside per-step
+    # events that then make up the timed total.
+    flush = None
+    if wl.nbytes < 2 * L2_BYTES:
+        flush = torch.zeros(2 * L2_BYTES // 4, dtype=torch.int32, device=dev)
+        sevs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
     with ClockSampler(local) as clk:
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
         t_start.record(stream)
         for i in range(K):
+            if flush is not None:
+                flush.add_(1)
+                sevs[i][0].record(stream)
             step(*evs[i])
+            if flush is not None:
+                sevs[i][1].record(stream)
         t_end.record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    total_ms = t_start.elapsed_time(t_end)
+    total_ms = t_start.elapsed_time(t_end) if flush is None else sum(a.elapsed_time(b) for a, b in sevs)
     kern_ms = float(np.mean([a.elapsed_time(b) for a, b in evs]))
     per_rank = None
     if world > 1:
@@ -651,7 +664,9 @@ def main():
             "algorithmic_bytes_per_gpu_step": nbytes,
             "table_entries": int(len(ents)),
             "fetch_status": int(ok_status),
-            "l2": "inputs >> 126 MB L2 (no flush needed)",
+            "l2": ("inputs >> 126 MB L2 (no flush needed)" if flush is None else
+                   f"inputs ({nbytes / 1e6:.0f} MB) fit the 126 MB L2: a {2 * L2_BYTES >> 20} MiB buffer is written "
+                   "between timed steps, outside the per-step events that make up ms_per_step"),
             "parallelism": f"shards x{world}" + ("" if world == 1 else (" + shared table over NVLink peer memory"
                                                                          if shared is not None else
                                                                          " + NCCL merge per step")),

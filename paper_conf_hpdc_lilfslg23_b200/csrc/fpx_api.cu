@@ -39,7 +39,13 @@ struct fpx_ctx {
   ListEntry* h_list = nullptr;
   uint32_t list_cap = 0;
   cudaEvent_t list_copied = nullptr;
+  // record-scan chunk counters (fpx_scan_records.cu Sched): kSchedSlots
+  // pairs, one per launch in turn, so that launches in flight on different
+  // streams never share one
+  unsigned int* d_sched = nullptr;
+  uint32_t sched_seq = 0;
 };
+constexpr uint32_t kSchedSlots = 64;
 
 namespace {
 
@@ -50,6 +56,17 @@ fpx_status cuda_err(cudaError_t e, const char* where) {
   std::lock_guard<std::mutex> lk(g_err_mu);
   snprintf(g_cuda_err, sizeof g_cuda_err, "%s: %s", where, cudaGetErrorString(e));
   return FPX_ERR_CUDA;
+}
+
+// The record scan's zeroed chunk counters (see fpx_ctx::d_sched).
+bool alloc_sched(fpx_ctx* h) {
+  const size_t b = 2 * sizeof(unsigned int) * kSchedSlots;
+  if (cudaMalloc(&h->d_sched, b) != cudaSuccess) {
+    cudaGetLastError();
+    h->d_sched = nullptr;
+    return false;
+  }
+  return cudaMemsetAsync(h->d_sched, 0, b, nullptr) == cudaSuccess;
 }
 
 #define CK(x)                                                  \
@@ -207,6 +224,10 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   h->tv.ctl = ctl;
   h->tv.flags = o.flags & FPX_OPT_NO_WARP_AGG;
   CK(launch_table_reset(h->tv, h->slots, nullptr));
+  if (!alloc_sched(h)) {
+    fpx_close(h);
+    return FPX_ERR_NOMEM;
+  }
   CK(cudaStreamSynchronize(nullptr));
   *out = h;
   return FPX_OK;
@@ -223,8 +244,9 @@ fpx_status fpx_scan_records(fpx_handle h, const fpx_rec_hdr* d_hdr, uint64_t n_r
   DeviceGuard g(h->device);
   if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  unsigned int* sched = h->d_sched + 2 * (h->sched_seq++ % kSchedSlots);
   CK(launch_scan_records(d_hdr, n_records, d_arena, arena_planes, base_index, mode, h->tv, h->num_sms, h->variant,
-                         s));
+                         sched, s));
   h->last_stream = s;
   return FPX_OK;
 }
@@ -518,6 +540,11 @@ fpx_status fpx_open_attached(int device, const fpx_ipc_table* t, fpx_handle* out
     delete h;
     return FPX_ERR_NOMEM;
   }
+  if (!alloc_sched(h)) {
+    fpx_close(h);
+    return FPX_ERR_NOMEM;
+  }
+  CK(cudaStreamSynchronize(nullptr));
   *out = h;
   return FPX_OK;
 }
@@ -543,7 +570,7 @@ fpx_status fpx_close(fpx_handle h) {
     if (h->d_list) cudaFree(h->d_list);
     if (h->list_copied) cudaEventDestroy(h->list_copied);
     for (void* p : {(void*)h->d_keys, (void*)h->d_counts, (void*)h->d_first, (void*)h->d_keys2, (void*)h->d_idx,
-                    (void*)h->d_idx2, (void*)h->d_n, h->d_temp})
+                    (void*)h->d_idx2, (void*)h->d_n, h->d_temp, (void*)h->d_sched})
       if (p) cudaFree(p);
   }
   delete h;

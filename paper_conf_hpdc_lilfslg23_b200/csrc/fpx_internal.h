@@ -56,10 +56,13 @@ struct alignas(16) ListEntry {
 static_assert(sizeof(ListEntry) == 64, "list entry is 64 B");
 
 // ---- launchers (fpx_scan_records.cu, fpx_scan_tensor.cu, fpx_table.cu) --------------------------------
-// variant 0 = TMA ring (default), 1 = register-staged LDG (FPX_OPT_SCAN_LDG ablation)
+// variant 0 = TMA ring (default), 1 = register-staged LDG (FPX_OPT_SCAN_LDG ablation).
+// sched_ctr: two zeroed u32 counters of the TMA kernel's dynamic tail, left
+// zeroed again when the launch completes (nullptr: static ranges only).
 cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena,
                                 uint64_t arena_planes, uint64_t base_index, uint32_t mode,
-                                const TableView& tv, int num_sms, uint32_t variant, cudaStream_t s);
+                                const TableView& tv, int num_sms, uint32_t variant, unsigned int* sched_ctr,
+                                cudaStream_t s);
 cudaError_t launch_scan_tensor(const void* d_ptr, uint64_t n_elems, uint32_t fmt, uint32_t site,
                                uint64_t base_index, const TableView& tv, int num_sms, cudaStream_t s);
 cudaError_t launch_scan_tensor_list(const ListEntry* d_entries, uint32_t n, uint64_t total_vec,

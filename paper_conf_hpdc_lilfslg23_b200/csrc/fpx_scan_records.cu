@@ -29,6 +29,7 @@
 // ring buys (profiles/).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdlib>
 
 #include "fpx_records.cuh"
@@ -329,10 +330,39 @@ __device__ __forceinline__ void consume_list(Witness& w, uint32_t b, uint32_t e,
   }
 }
 
+// Load balance of the record scan.  Every warp first scans a static
+// contiguous range (recs_per_warp records, ~3/4 of the trace); the rest,
+// [dyn0, n), is cut into chunks that warps claim with an atomicAdd on ctr[0]
+// as they run out of work: nbig chunks of `chunk` records over [dyn0, dyn1),
+// then one-tile chunks over [dyn1, n) (about two per warp), so that the last
+// claims are short and the warps finish within a tile of each other.  Equal record counts are not
+// equal work: FP64-heavy stretches of a trace carry twice the bytes and
+// exception storms take the exact path, so static ranges alone leave the SMs
+// idle for 10-15 % of a C2 launch while the slowest warps finish
+// (tools/warp_times.py).  ctr[1] counts finished warps; the last one resets
+// both counters, so each launch finds them at zero (the API gives concurrent
+// launches different counter pairs).  nchunks = 0: static ranges only.
+constexpr uint64_t kDynMinTiles = 16;  // dynamic tail only from 16 tiles per warp up
+constexpr uint32_t kDynChunk = 256;     // records per claimed chunk (8 tiles)
+constexpr int kStaticPct = 75;          // share of the trace in static ranges
+struct Sched {
+  unsigned int* ctr;
+  uint64_t dyn0, dyn1;
+  uint32_t chunk, nbig, nchunks, nwarps;
+};
+
+#ifdef FPX_WARP_TIMES
+// Diagnostics build only (tools/warp_times.py): %globaltimer at each warp's
+// start and end of the last record-scan launch, to measure load imbalance.
+constexpr int kMaxWarpTimes = 148 * 32;
+__device__ unsigned long long g_warp_t0[kMaxWarpTimes], g_warp_t1[kMaxWarpTimes];
+#endif
+
 template <int MODE, class C>
 __global__ void __launch_bounds__(C::WARPS * 32, 1)
 k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __restrict__ arena,
-                   uint64_t arena_planes, uint64_t base_index, uint64_t recs_per_warp, const TableView tv) {
+                   uint64_t arena_planes, uint64_t base_index, uint64_t recs_per_warp, const Sched sch,
+                   const TableView tv) {
   constexpr int STAGES = C::STAGES, PLANES = C::PLANES;
   static_assert(PLANES <= 64, "stage sizes keep the byte fields of the packed scan exact");
   extern __shared__ __align__(128) uint8_t smem_raw[];
@@ -344,7 +374,14 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   const uint64_t gw = blockIdx.x * (uint64_t)C::WARPS + warp;
   const uint64_t start = gw * recs_per_warp;
   if (start >= n) return;  // warp-uniform; no block-wide barriers below this line
+#ifdef FPX_WARP_TIMES
+  if (lane == 0 && gw < kMaxWarpTimes) g_warp_t0[gw] = globaltimer_ns();
+#endif
   const uint64_t end = min(n, start + recs_per_warp);
+  // dynamic tail (Sched): the chunk this warp takes after its current range,
+  // claimed one range ahead so the atomic's latency stays off the critical path
+  uint32_t claim = 0;
+  if (sch.nchunks != 0u && lane == 0) claim = atomicAdd(sch.ctr, 1u);
   const uint32_t* __restrict__ lane_base = arena + lane;
   const uint64_t policy = policy_evict_first();
   const uint32_t g = (uint32_t)lane >> 3, q = (uint32_t)lane & 7u;
@@ -360,6 +397,18 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   // this warp's range (< 2^31, checked at launch: 32-bit lane tests)
   uint64_t cursor = start;
   uint32_t rem = (uint32_t)(end - start);
+  // at the end of a range: move into the claimed chunk and claim the next
+  auto next_range = [&]() {
+    if (rem == 0u && sch.nchunks != 0u) {
+      const uint32_t c = __shfl_sync(FULL, claim, 0);
+      if (c < sch.nchunks) {
+        cursor = c < sch.nbig ? sch.dyn0 + (uint64_t)c * sch.chunk : sch.dyn1 + (uint64_t)(c - sch.nbig) * TILE;
+        rem = (uint32_t)min((uint64_t)(c < sch.nbig ? sch.chunk : TILE), n - cursor);
+        if (lane == 0) claim = atomicAdd(sch.ctr, 1u);
+      }
+    }
+  };
+  next_range();
   uint4 h = make_uint4(0, 0, 0, 0);
   if ((uint32_t)lane < rem) h = ld_stream4(hdr + cursor + lane);
 
@@ -462,6 +511,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     // advance and prefetch the next tile's headers
     cursor += k;
     rem -= k;
+    next_range();
     h = make_uint4(0, 0, 0, 0);
     if ((uint32_t)lane < rem) h = ld_stream4(hdr + cursor + lane);
   };
@@ -474,7 +524,17 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const int s = (int)(i % STAGES);
     produce((int)((i + STAGES - 1) % STAGES));
     const StageMeta& m = sm.meta[s];
-    if (m.k == 0u) break;
+    if (m.k == 0u) {
+#ifdef FPX_WARP_TIMES
+      if (lane == 0 && gw < kMaxWarpTimes) g_warp_t1[gw] = globaltimer_ns();
+#endif
+      // the last warp out re-arms the launch's chunk counters for reuse
+      if (sch.nchunks != 0u && lane == 0 && atomicAdd(sch.ctr + 1, 1u) == sch.nwarps - 1u) {
+        atomicExch(sch.ctr, 0u);
+        atomicExch(sch.ctr + 1, 0u);
+      }
+      break;
+    }
     mbar_wait(&sm.bar[s], (phase >> s) & 1u);
     phase ^= 1u << s;
 
@@ -523,7 +583,8 @@ static_assert(sizeof(WarpSmem<Ring2>) % 128 == 0 && ring_smem<Ring0>() <= 227 * 
 
 template <int MODE, class C>
 cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uint64_t arena_planes, uint64_t base_index,
-                        const TableView& tv, int num_sms, cudaStream_t s) {
+                        const TableView& tv, int num_sms, unsigned int* sched_ctr, bool tile_tail, int static_pct,
+                        cudaStream_t s) {
   static bool attr_set[64] = {};  // per device
   int dev = 0;
   cudaGetDevice(&dev);
@@ -536,12 +597,30 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
   // one CTA per SM; each warp a contiguous range of records (whole tiles of 32
   // where possible, so that ranges stay 512-B aligned in the header array)
   const uint64_t warps = (uint64_t)num_sms * C::WARPS;
-  uint64_t per = (n + warps - 1) / warps;
-  per = (per + TILE - 1) / TILE * TILE;
+  Sched sch{sched_ctr, n, n, 0u, 0u, 0u, 0u};
+  uint64_t per, blocks;
+  if (sched_ctr != nullptr && n >= warps * TILE * kDynMinTiles) {
+    // static ranges: 3/4 of the trace in whole tiles; the rest in chunks
+    per = n / 100 * (uint64_t)static_pct / warps / TILE * TILE;
+    sch.dyn0 = per * warps;
+    sch.chunk = kDynChunk;
+    const uint64_t rest = n - sch.dyn0, small = tile_tail ? std::min<uint64_t>(rest, warps * 2 * TILE) : 0;
+    const uint64_t nbig = (rest - small) / kDynChunk;
+    sch.dyn1 = sch.dyn0 + nbig * kDynChunk;
+    const uint64_t nch = nbig + (n - sch.dyn1 + TILE - 1) / TILE;
+    if (nch >= (1ull << 31)) return cudaErrorInvalidValue;
+    sch.nbig = (uint32_t)nbig;
+    sch.nchunks = (uint32_t)nch;
+    sch.nwarps = (uint32_t)warps;
+    blocks = (uint64_t)num_sms;
+  } else {
+    per = (n + warps - 1) / warps;
+    per = (per + TILE - 1) / TILE * TILE;
+    blocks = ((n + per - 1) / per + C::WARPS - 1) / C::WARPS;
+  }
   if (per >= (1ull << 31)) return cudaErrorInvalidValue;  // the kernel counts a warp's records in 32 bits
-  const uint64_t blocks = ((n + per - 1) / per + C::WARPS - 1) / C::WARPS;
   k_scan_records_tma<MODE, C><<<(unsigned)blocks, C::WARPS * 32, ring_smem<C>(), s>>>(hdr, n, arena, arena_planes,
-                                                                                      base_index, per, tv);
+                                                                                      base_index, per, sch, tv);
   return cudaGetLastError();
 }
 
@@ -687,7 +766,7 @@ k_scan_records_ldg(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 template <int MODE>
 cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena, uint64_t arena_planes,
                              uint64_t base_index, const TableView& tv, int num_sms, uint32_t variant,
-                             cudaStream_t s) {
+                             unsigned int* sched_ctr, cudaStream_t s) {
   if (variant == 1u) {
     const uint64_t tiles = (n + TILE - 1) / TILE;
     uint64_t blocks = (tiles + LDG_WARPS - 1) / LDG_WARPS;
@@ -714,12 +793,26 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   // NaN storm S2 by 11 % (its exact path wants more warps): the common case
   // decides.
   if (ring < 0) ring = n <= (uint64_t)num_sms * 24 * TILE ? 3 : 1;
+  // FPX_SCHED (environment, A/B only): 0 = static ranges, 2 = no one-tile
+  // chunks at the end; default 1
+  static int sched_env = -2;
+  if (sched_env == -2) {
+    const char* e = getenv("FPX_SCHED");
+    sched_env = e ? atoi(e) : 1;
+  }
+  if (sched_env == 0) sched_ctr = nullptr;
+  const bool tile_tail = sched_env != 2;
+  static int static_pct = -1;  // FPX_STATIC_PCT (environment, A/B only): share of static ranges
+  if (static_pct < 0) {
+    const char* e = getenv("FPX_STATIC_PCT");
+    static_pct = e ? std::max(0, std::min(100, atoi(e))) : kStaticPct;
+  }
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   switch (ring) {
-    case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
-    case 2: return launch_ring<MODE, Ring2>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
-    case 3: return launch_ring<MODE, Ring3>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
-    default: return launch_ring<MODE, Ring0>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, s);
+    case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, tile_tail, static_pct, s);
+    case 2: return launch_ring<MODE, Ring2>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, tile_tail, static_pct, s);
+    case 3: return launch_ring<MODE, Ring3>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, tile_tail, static_pct, s);
+    default: return launch_ring<MODE, Ring0>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, tile_tail, static_pct, s);
   }
 }
 
@@ -727,12 +820,24 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
 
 cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena, uint64_t arena_planes,
                                 uint64_t base_index, uint32_t mode, const TableView& tv, int num_sms, uint32_t variant,
-                                cudaStream_t s) {
+                                unsigned int* sched_ctr, cudaStream_t s) {
   if (mode == FPX_MODE_DEST)
-    return launch_records_t<FPX_MODE_DEST>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, s);
+    return launch_records_t<FPX_MODE_DEST>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, sched_ctr, s);
   if (mode == FPX_MODE_FLOW)
-    return launch_records_t<FPX_MODE_FLOW>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, s);
-  return launch_records_t<FPX_MODE_FLOW_DETAIL>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, s);
+    return launch_records_t<FPX_MODE_FLOW>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, sched_ctr, s);
+  return launch_records_t<FPX_MODE_FLOW_DETAIL>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, sched_ctr, s);
 }
 
 }  // namespace fpx
+
+#ifdef FPX_WARP_TIMES
+// Copies the per-warp start / end times of the last record-scan launch
+// (diagnostics build only; not part of include/fpx.h).
+extern "C" __attribute__((visibility("default"))) int fpx_debug_warp_times(unsigned long long* t0,
+                                                                            unsigned long long* t1, int n) {
+  if (n > fpx::kMaxWarpTimes) n = fpx::kMaxWarpTimes;
+  if (cudaMemcpyFromSymbol(t0, fpx::g_warp_t0, n * sizeof(unsigned long long)) != cudaSuccess) return -1;
+  if (cudaMemcpyFromSymbol(t1, fpx::g_warp_t1, n * sizeof(unsigned long long)) != cudaSuccess) return -1;
+  return n;
+}
+#endif

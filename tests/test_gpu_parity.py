@@ -442,3 +442,53 @@ def test_scan_tensors_one_launch(fpx):
                                    torch.bfloat16: BF16}[t.dtype], site=site, base_index=b)
     assert_same(got, ref.entries())
     assert_same(single, ref.entries())
+
+
+# ---------------------------------------------------------------------------
+# Dynamic tail of the record scan (fpx_scan_records.cu Sched): from 16 tiles per
+# warp up, warps scan 3/4 of the trace in static ranges and claim the rest in
+# 256-record chunks.  Sizes here reach that regime (>= 148 * 20 * 512 records)
+# with a ragged last chunk; the oracle still finishes in seconds.
+@pytest.mark.parametrize("name,recipe,mode,n", [
+    ("mix", fpxgen.RECIPE_MIX, DEST, 1_600_037),
+    ("flow", fpxgen.RECIPE_FLOW, FLOW, 1_550_011),
+    ("packed", fpxgen.RECIPE_PACKED, DEST, 1_520_129),
+], ids=["mix", "flow", "packed"])
+def test_dynamic_tail_parity(fpx, name, recipe, mode, n):
+    p = fpxgen.Params(seed=0x5EED0100 + recipe, n_records=n, n_sites=3_000, recipe=recipe, p_fp64=0.5)
+    hdr, arena = fpxgen.generate_host(p)
+    inj, w = fpxgen.plan_injections(p, 3_000, flow=(recipe == fpxgen.RECIPE_FLOW))
+    fpxgen.apply_host(w, hdr, arena)
+    base = 3 * 10**9
+    got, st, stats = gpu_scan(fpx, hdr, arena, base=base, mode=mode)
+    assert st == fpx.OK and stats.bad_records == 0
+    assert_same(got, oracle_scan(hdr, arena, base, mode).entries())
+    assert table_dict(got) == expected_from_injections(hdr, inj, base, mode)
+
+
+def test_dynamic_tail_relaunch_and_streams(fpx):
+    """The chunk counters re-arm themselves: back-to-back launches without a
+    reset add up exactly (count x 3, same first index), and launches in
+    flight on two streams at once (different counter pairs) do too."""
+    n = 1_600_001
+    p = fpxgen.Params(seed=41, n_records=n, n_sites=500, recipe=fpxgen.RECIPE_MIX, p_fp64=0.5)
+    hdr, arena = fpxgen.generate_host(p)
+    _, w = fpxgen.plan_injections(p, 2_000)
+    fpxgen.apply_host(w, hdr, arena)
+    exp = table_dict(oracle_scan(hdr, arena, 0, DEST).entries())
+    d_hdr, d_arena = to_dev(hdr, arena)
+    planes = arena.size // 32
+    with fpx.Handle(0) as h:
+        for _ in range(3):
+            h.scan_records(d_hdr, d_arena, base_index=0, n_records=n, arena_planes=planes)
+        got = table_dict(h.fetch())
+        assert got == {k: [3 * c, f] for k, (c, f) in exp.items()}
+        h.reset()
+        s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+        torch.cuda.synchronize()
+        for _ in range(2):
+            for s in (s1, s2):
+                h.scan_records(d_hdr, d_arena, base_index=0, n_records=n, arena_planes=planes, stream=s)
+        torch.cuda.synchronize()
+        got = table_dict(h.fetch())
+        assert got == {k: [4 * c, f] for k, (c, f) in exp.items()}

@@ -1,0 +1,70 @@
+"""Load imbalance of the record scan: per-warp start / end times (%globaltimer)
+of one launch, from a diagnostics build of libfpx.so (-DFPX_WARP_TIMES).
+
+    python tools/warp_times.py [config ...]      # default: c2 c3 c4a c5
+
+Builds build/libfpx_wt.so, scans each bench config (same trace as bench.py)
+a few times and prints, for the last launch: the kernel span (last end - first
+start), the warp durations (min / median / max) and the end-time spread — the
+share of the span the SMs spend idle waiting for the slowest warp."""
+import ctypes
+import os
+import subprocess
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+LIB = os.path.join(ROOT, "build", "libfpx_wt.so")
+CSRC = os.path.join(ROOT, "paper_conf_hpdc_lilfslg23_b200", "csrc")
+SRC = [os.path.join(CSRC, f) for f in ("fpx_api.cu", "fpx_scan_records.cu", "fpx_scan_tensor.cu", "fpx_table.cu")]
+
+os.makedirs(os.path.dirname(LIB), exist_ok=True)
+subprocess.run(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-Xcompiler",
+                "-fPIC,-O3", "-shared", "-I" + os.path.join(ROOT, "include"), "-DFPX_WARP_TIMES", *SRC, "-o", LIB],
+               check=True)
+os.environ["FPX_LIB"] = LIB
+
+import torch  # noqa: E402
+
+import bench  # noqa: E402
+from paper_conf_hpdc_lilfslg23_b200 import fpx  # noqa: E402
+
+wt = ctypes.CDLL(LIB)
+wt.fpx_debug_warp_times.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int]
+NW = 148 * 32
+
+for name in sys.argv[1:] or ["c2", "c3", "c4a", "c5"]:
+    cfg = dict(bench.CONFIGS[name])
+    wl = bench.RecordsWorkload(cfg, 0, bench.config_seed(name), "tma")
+    stream = torch.cuda.current_stream()
+    h = fpx.Handle(0)
+    t0 = np.zeros(NW, dtype=np.uint64)
+    t1 = np.zeros(NW, dtype=np.uint64)
+    spans = []
+    for rep in range(6):
+        h.reset(stream=stream)
+        wl.scan(h, stream)
+        torch.cuda.synchronize()
+        n = wt.fpx_debug_warp_times(t0.ctypes.data, t1.ctypes.data, NW)
+        live = (t0[:n] != 0) & (t1[:n] >= t0[:n])
+        a, b = t0[:n][live].astype(np.int64), t1[:n][live].astype(np.int64)
+        if rep >= 2:
+            spans.append((a, b))
+        t0[:] = 0
+        t1[:] = 0
+    for a, b in spans[-2:]:
+        s0 = a.min()
+        span = b.max() - s0
+        dur = b - a
+        ends = np.sort(b - s0)
+        idle = 1.0 - dur.sum() / (len(dur) * span)
+        print(f"{name}: warps {len(dur)} span {span / 1e3:.1f} us | warp dur min/med/max "
+              f"{dur.min() / 1e3:.1f}/{np.median(dur) / 1e3:.1f}/{dur.max() / 1e3:.1f} us | start spread "
+              f"{(a.max() - s0) / 1e3:.1f} us | end p10/p50/p90/max {ends[len(ends) // 10] / 1e3:.1f}/"
+              f"{ends[len(ends) // 2] / 1e3:.1f}/{ends[9 * len(ends) // 10] / 1e3:.1f}/{ends[-1] / 1e3:.1f} us | "
+              f"idle share {100 * idle:.1f} %", flush=True)
+    h.close()
+    del wl
+    torch.cuda.empty_cache()
