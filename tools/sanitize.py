@@ -1,6 +1,6 @@
 """Small scans of every kernel family for compute-sanitizer (memcheck,
 racecheck, synccheck): DEST / FLOW / FLOW_DETAIL record scans (TMA ring and
-LDG), a storm trace (exact path + table atomics), tensor scans with ragged
+LDG), the record scan's dynamic tail, a storm trace (exact path + table atomics), tensor scans with ragged
 heads / tails, fetch / FETCH_NEW / reset / merge paths."""
 import os
 import sys
@@ -29,6 +29,17 @@ for recipe, mode in ((fpxgen.RECIPE_MIX, 0), (fpxgen.RECIPE_FLOW, 1), (fpxgen.RE
             h.reset()
             h.merge_device(k, c, f)
             assert len(h.fetch()) == len(e) == len(n)
+# the record scan's dynamic tail (>= 148 x 20 x 512 records): chunks claimed by
+# atomics, counters re-armed by the last warp; two launches back to back
+p = fpxgen.Params(seed=11, n_records=1_520_011, n_sites=300, recipe=fpxgen.RECIPE_MIX, p_fp64=0.5)
+hdr, arena, planes = fpxgen.generate_device(p)
+_, w = fpxgen.plan_injections(p, 500)
+fpxgen.apply_device(w, hdr, arena)
+with fpx.Handle(0) as h:
+    for _ in range(2):
+        h.scan_records(hdr, arena, arena_planes=planes)
+    h.fetch()
+del hdr, arena
 p = fpxgen.Params(seed=9, n_records=5000, n_sites=20, recipe=fpxgen.RECIPE_STRESS, dense_nan=1.0)
 hdr, arena, planes = fpxgen.generate_device(p)
 with fpx.Handle(0, table_log2_slots=5) as h:
