@@ -345,6 +345,11 @@ __device__ __forceinline__ void consume_list(Witness& w, uint32_t b, uint32_t e,
 constexpr uint64_t kDynMinTiles = 16;  // dynamic tail only from 16 tiles per warp up
 constexpr uint32_t kDynChunk = 256;     // records per claimed chunk (8 tiles)
 constexpr int kStaticPct = 75;          // share of the trace in static ranges
+constexpr uint32_t kTailTiles = 8;      // one-tile chunks at the end, per warp
+struct SchedCfg {
+  int static_pct;
+  uint32_t chunk, tail_tiles;
+};
 struct Sched {
   unsigned int* ctr;
   uint64_t dyn0, dyn1;
@@ -583,7 +588,7 @@ static_assert(sizeof(WarpSmem<Ring2>) % 128 == 0 && ring_smem<Ring0>() <= 227 * 
 
 template <int MODE, class C>
 cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uint64_t arena_planes, uint64_t base_index,
-                        const TableView& tv, int num_sms, unsigned int* sched_ctr, bool tile_tail, int static_pct,
+                        const TableView& tv, int num_sms, unsigned int* sched_ctr, const SchedCfg& scfg,
                         cudaStream_t s) {
   static bool attr_set[64] = {};  // per device
   int dev = 0;
@@ -601,12 +606,12 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
   uint64_t per, blocks;
   if (sched_ctr != nullptr && n >= warps * TILE * kDynMinTiles) {
     // static ranges: 3/4 of the trace in whole tiles; the rest in chunks
-    per = n / 100 * (uint64_t)static_pct / warps / TILE * TILE;
+    per = n / 100 * (uint64_t)scfg.static_pct / warps / TILE * TILE;
     sch.dyn0 = per * warps;
-    sch.chunk = kDynChunk;
-    const uint64_t rest = n - sch.dyn0, small = tile_tail ? std::min<uint64_t>(rest, warps * 2 * TILE) : 0;
-    const uint64_t nbig = (rest - small) / kDynChunk;
-    sch.dyn1 = sch.dyn0 + nbig * kDynChunk;
+    sch.chunk = scfg.chunk;
+    const uint64_t rest = n - sch.dyn0, small = std::min<uint64_t>(rest, warps * scfg.tail_tiles * TILE);
+    const uint64_t nbig = (rest - small) / scfg.chunk;
+    sch.dyn1 = sch.dyn0 + nbig * scfg.chunk;
     const uint64_t nch = nbig + (n - sch.dyn1 + TILE - 1) / TILE;
     if (nch >= (1ull << 31)) return cudaErrorInvalidValue;
     sch.nbig = (uint32_t)nbig;
@@ -801,18 +806,25 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
     sched_env = e ? atoi(e) : 1;
   }
   if (sched_env == 0) sched_ctr = nullptr;
-  const bool tile_tail = sched_env != 2;
-  static int static_pct = -1;  // FPX_STATIC_PCT (environment, A/B only): share of static ranges
+  // FPX_STATIC_PCT / FPX_DYN_CHUNK / FPX_TAIL_TILES (environment, A/B only):
+  // share of static ranges, records per big chunk, one-tile chunks per warp
+  static int static_pct = -1, dyn_chunk = -1, tail_tiles = -1;
   if (static_pct < 0) {
     const char* e = getenv("FPX_STATIC_PCT");
     static_pct = e ? std::max(0, std::min(100, atoi(e))) : kStaticPct;
+    e = getenv("FPX_DYN_CHUNK");
+    dyn_chunk = e ? std::max(1, atoi(e) / TILE) * TILE : (int)kDynChunk;
+    e = getenv("FPX_TAIL_TILES");
+    tail_tiles = e ? std::max(0, atoi(e)) : (int)kTailTiles;
   }
+  if (sched_env == 2) tail_tiles = 0;
+  const SchedCfg scfg{static_pct, (uint32_t)dyn_chunk, (uint32_t)tail_tiles};
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   switch (ring) {
-    case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, tile_tail, static_pct, s);
-    case 2: return launch_ring<MODE, Ring2>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, tile_tail, static_pct, s);
-    case 3: return launch_ring<MODE, Ring3>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, tile_tail, static_pct, s);
-    default: return launch_ring<MODE, Ring0>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, tile_tail, static_pct, s);
+    case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, s);
+    case 2: return launch_ring<MODE, Ring2>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, s);
+    case 3: return launch_ring<MODE, Ring3>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, s);
+    default: return launch_ring<MODE, Ring0>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, s);
   }
 }
 
