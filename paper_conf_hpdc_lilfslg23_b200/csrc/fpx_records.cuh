@@ -83,6 +83,33 @@ __device__ __forceinline__ void for_each_dest_kind(uint32_t op, uint32_t fmt, ui
   }
 }
 
+// Table 2's state of one lane-value of a scalar FP32 / FP64 record (FLOW
+// modes): S = the most severe class among the pre-execution sources (NaN > INF
+// > SUB, R5), src = the lowest-index source holding it (R21); D = the
+// destination kind (dest_kind).  Returns flow << 2 | kind, or CODE_NONE.
+__device__ __forceinline__ int flow_code(uint32_t op, uint32_t fmt, uint32_t nsrc, uint32_t dw, bool have_div,
+                                         const uint32_t* dv, const uint32_t* sv, int& S, uint32_t& src) {
+  S = CODE_NONE;
+  src = 0;
+  int sev = 0;
+#pragma unroll
+  for (uint32_t k = 0; k < 3; ++k) {
+    if (k >= nsrc) break;
+    const uint32_t c = fmt == FPX_FP64 ? cls_fp64(sv[2 * k], sv[2 * k + 1]) : cls_fp32(sv[k]);
+    const int sv_ = c == CLS_NAN ? 3 : c == CLS_INF ? 2 : c == CLS_SUB ? 1 : 0;
+    if (sv_ > sev) { sev = sv_; S = kind_of_cls(c); src = k; }
+  }
+  int D = CODE_NONE;
+  if (dw != 0u) {
+    if (fmt == FPX_FP64) D = dest_kind(op, fmt, dv[0], dv[1], have_div, sv[0], sv[1], sv[2], sv[3]);
+    else D = dest_kind(op, fmt, dv[0], 0u, have_div, sv[0], 0u, sv[1], 0u);
+  }
+  if (D >= 0 && S < 0) return (FPX_GEN << 2) | D;
+  if (D >= 0) return (FPX_PROP << 2) | D;
+  if (S >= 0) return (FPX_KILL << 2) | S;
+  return CODE_NONE;
+}
+
 // Exact evaluation of one record for this lane (both modes).  Returns the
 // bitmask of event codes held by this lane; codes / evm describe per-value
 // codes for count_of().
@@ -117,26 +144,9 @@ __device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t
     });
     return cm;
   } else {
-    // Analyzer: S = most severe class among the pre-execution sources; src =
-    // the lowest-index source holding it (R21).
-    int S = CODE_NONE, sev = 0;
-    uint32_t src = 0;
-#pragma unroll
-    for (uint32_t k = 0; k < 3; ++k) {
-      if (k >= nsrc) break;
-      const uint32_t c = fmt == FPX_FP64 ? cls_fp64(sv[2 * k], sv[2 * k + 1]) : cls_fp32(sv[k]);
-      const int sv_ = c == CLS_NAN ? 3 : c == CLS_INF ? 2 : c == CLS_SUB ? 1 : 0;
-      if (sv_ > sev) { sev = sv_; S = kind_of_cls(c); src = k; }
-    }
-    int D = CODE_NONE;
-    if (dw != 0u) {
-      if (fmt == FPX_FP64) D = dest_kind(op, fmt, dv[0], dv[1], have_div, sv[0], sv[1], sv[2], sv[3]);
-      else D = dest_kind(op, fmt, dv[0], 0u, have_div, sv[0], 0u, sv[1], 0u);
-    }
-    int code = CODE_NONE;
-    if (D >= 0 && S < 0) code = (FPX_GEN << 2) | D;
-    else if (D >= 0) code = (FPX_PROP << 2) | D;
-    else if (S >= 0) code = (FPX_KILL << 2) | S;
+    int S;
+    uint32_t src;
+    int code = flow_code(op, fmt, nsrc, dw, have_div, dv, sv, S, src);
     if (code < 0) return 0u;
     // FLOW_DETAIL: detail = 1 + src, | CMP for Table 1's control-flow opcodes (R22)
     if (MODE == FPX_MODE_FLOW_DETAIL && S >= 0) {
@@ -341,7 +351,11 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
 // (exact_tile_transposed; a tile mixing formats runs each present format's
 // class loop in turn, still far cheaper than walking the records), the
 // analyzer modes and the no-aggregation ablation record by record
-// (exact_tile_records).  A/B in profiles/r1/ab_producer.txt (ab9-ab16).
+// (exact_tile_records).  A transposed FLOW path (lane groups per record,
+// (destination, source) severity bins) was tried and lost 1.7-2.3x on
+// storm-heavy FLOW traces: FLOW tiles hold ~10 records, so most lanes idle,
+// and per-record operand counts and formats diverge inside the loop
+// (profiles/r1/ab_sched.txt).  A/B in profiles/r1/ab_producer.txt (ab9-ab16).
 template <int MODE, typename Needed>
 __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
                                             const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
