@@ -221,7 +221,11 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out);
  * bits, enum ranges, planes outside the arena, invalid site, and in the FLOW
  * modes records other than scalar FP32/FP64) are counted and skipped.
  * n_records == 0 is a no-op.  Buffers must stay valid until the stream passes
- * the scan.  Errors: FPX_ERR_INVALID, FPX_ERR_CUDA. */
+ * the scan.  Large scans balance work across warps with two device counters
+ * owned by the handle; a handle keeps 64 counter pairs and hands them out in
+ * turn, so at most 64 record scans of one handle may be in flight at once on
+ * different streams (scans on one stream are always safe).  Errors:
+ * FPX_ERR_INVALID, FPX_ERR_CUDA. */
 fpx_status fpx_scan_records(fpx_handle h, const fpx_rec_hdr* d_hdr, uint64_t n_records,
                             const uint32_t* d_arena, uint64_t arena_planes,
                             uint64_t base_index, uint32_t mode, void* stream);
