@@ -332,7 +332,23 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
   uint32_t present = 0u;
 #pragma unroll
   for (int kd = 0; kd < 4; ++kd) present |= ((cnt >> (16 * kd)) & 0xFFFFu) ? 1u << kd : 0u;
-  uint32_t all = __reduce_or_sync(FULL, present);
+  // Group per kind, then issue every group's table update at once: a leader
+  // parks its sums (one per kind it leads) and the updates of different kinds
+  // and records run in parallel instead of one warp-wide round per kind (C1
+  // +11 %).  A single kind (storms) updates right away (S2 -2 % otherwise).
+  uint32_t all = __reduce_or_sync(FULL, present), lead = 0u;
+  if (__popc(all) == 1) {
+    const uint32_t kd = (uint32_t)(__ffs(all) - 1);
+    const bool has = present != 0u;
+    const unsigned long long key = has ? make_key(h.x, fmt, kd) : FPX_KEY_EMPTY - (unsigned long long)lane;
+    const uint32_t peers = __match_any_sync(FULL, key);
+    if (has) {
+      const uint32_t sum = __reduce_add_sync(peers, (uint32_t)((cnt >> (16 * kd)) & 0xFFFFu));
+      if ((uint32_t)lane == (uint32_t)(__ffs(peers) - 1)) table_add(tv, key, sum, gidx0 + (uint64_t)lane);
+    }
+    return;
+  }
+  unsigned long long sums = 0ull;  // 16 bits per kind led by this lane
   while (all) {
     const uint32_t kd = (uint32_t)(__ffs(all) - 1);
     all &= all - 1u;
@@ -342,8 +358,16 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
     const uint32_t peers = __match_any_sync(FULL, key);
     if (has) {
       const uint32_t sum = __reduce_add_sync(peers, (uint32_t)((cnt >> (16 * kd)) & 0xFFFFu));
-      if ((uint32_t)lane == (uint32_t)(__ffs(peers) - 1)) table_add(tv, key, sum, gidx0 + (uint64_t)lane);
+      if ((uint32_t)lane == (uint32_t)(__ffs(peers) - 1)) {
+        lead |= 1u << kd;
+        sums |= (unsigned long long)sum << (16 * kd);
+      }
     }
+  }
+  while (lead) {
+    const uint32_t kd = (uint32_t)(__ffs(lead) - 1);
+    lead &= lead - 1u;
+    table_add(tv, make_key(h.x, fmt, kd), (sums >> (16 * kd)) & 0xFFFFu, gidx0 + (uint64_t)lane);
   }
 }
 
