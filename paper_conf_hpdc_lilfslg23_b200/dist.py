@@ -122,16 +122,33 @@ class SharedTable:
                 self.handle.close()
             raise RuntimeError(f"shared table unavailable: {self.error}")
 
+    # Ordering between ranks.  Under NCCL it is stream-ordered: a one-element
+    # all_reduce enqueued on the scan stream completes on no rank before every
+    # rank has reached it, so "home cleared the table" and "every rank's scan
+    # finished" become device-side dependencies with no host round trip per
+    # step.  Under gloo (CPU tests, ranks sharing one GPU) the host waits for
+    # the stream and meets the other ranks at a barrier.
+    def _sync(self, stream):
+        s = torch.cuda.current_stream() if stream is None else stream
+        if dist.get_backend(self.group) == "nccl":
+            if getattr(self, "_tok", None) is None:
+                self._tok = torch.zeros(1, dtype=torch.int32, device=torch.cuda.current_device())
+            with torch.cuda.stream(s):
+                dist.all_reduce(self._tok, group=self.group)
+        else:
+            s.synchronize()
+            dist.barrier(group=self.group)
+
     def reset(self, stream=None):
-        """Home clears the table; everyone waits for it before scanning again."""
+        """Home clears the table; no rank scans again before the clear is done."""
         if self.rank == self.home:
             self.handle.reset(stream=stream)
-            torch.cuda.current_stream().synchronize() if stream is None else stream.synchronize()
-        dist.barrier(group=self.group)
+        self._sync(stream)
 
     def finish(self, stream=None):
-        (torch.cuda.current_stream() if stream is None else stream).synchronize()
-        dist.barrier(group=self.group)
+        """Every rank's inserts have landed in the home table: on return (gloo)
+        or in `stream` order (NCCL; fetch() on the home rank waits for it)."""
+        self._sync(stream)
 
     def fetch(self):
         assert self.rank == self.home, "the home rank owns the shared table"
