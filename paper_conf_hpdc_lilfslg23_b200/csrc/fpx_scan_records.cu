@@ -331,17 +331,18 @@ __device__ __forceinline__ void consume_list(Witness& w, uint32_t b, uint32_t e,
 }
 
 // Load balance of the record scan.  Every warp first scans a static
-// contiguous range (recs_per_warp records, ~3/4 of the trace); the rest,
+// contiguous range (recs_per_warp records, 3/4 of the trace); the rest,
 // [dyn0, n), is cut into chunks that warps claim with an atomicAdd on ctr[0]
 // as they run out of work: nbig chunks of `chunk` records over [dyn0, dyn1),
-// then one-tile chunks over [dyn1, n) (about two per warp), so that the last
-// claims are short and the warps finish within a tile of each other.  Equal record counts are not
-// equal work: FP64-heavy stretches of a trace carry twice the bytes and
-// exception storms take the exact path, so static ranges alone leave the SMs
-// idle for 10-15 % of a C2 launch while the slowest warps finish
-// (tools/warp_times.py).  ctr[1] counts finished warps; the last one resets
-// both counters, so each launch finds them at zero (the API gives concurrent
-// launches different counter pairs).  nchunks = 0: static ranges only.
+// then one-tile chunks over [dyn1, n) (kTailTiles per warp), so that the last
+// claims are short and the warps finish within a tile or two of each other.
+// Equal record counts are not equal work: FP64-heavy stretches of a trace
+// carry twice the bytes and exception storms take the exact path, so static
+// ranges alone leave the SMs idle for 12-14 % of a C2 launch while the
+// slowest warps finish (tools/warp_times.py, profiles/r1/ab_sched.txt).
+// ctr[1] counts finished warps; the last one resets both counters, so each
+// launch finds them at zero (the API gives concurrent launches different
+// counter pairs).  nchunks = 0: static ranges only.
 constexpr uint64_t kDynMinTiles = 16;  // dynamic tail only from 16 tiles per warp up
 constexpr uint32_t kDynChunk = 256;     // records per claimed chunk (8 tiles)
 constexpr int kStaticPct = 75;          // share of the trace in static ranges
