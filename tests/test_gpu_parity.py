@@ -446,14 +446,20 @@ def test_scan_tensors_one_launch(fpx):
 
 # ---------------------------------------------------------------------------
 # Dynamic tail of the record scan (fpx_scan_records.cu Sched): from 16 tiles per
-# warp up, warps scan 3/4 of the trace in static ranges and claim the rest in
-# 256-record chunks.  Sizes here reach that regime (>= 148 * 20 * 512 records)
-# with a ragged last chunk; the oracle still finishes in seconds.
+# warp up (148 * 20 * 512 = 1,515,520 records), warps scan 3/4 of the trace in
+# static ranges and claim the rest: 256-record chunks, then 8 one-tile chunks
+# per warp.  ~1.5e6 records: the rest fits the one-tile chunks alone; ~4e6:
+# both kinds of chunk; the threshold itself and one record below it (static
+# ranges only); ragged last chunks throughout.  The oracle finishes in seconds.
 @pytest.mark.parametrize("name,recipe,mode,n", [
     ("mix", fpxgen.RECIPE_MIX, DEST, 1_600_037),
     ("flow", fpxgen.RECIPE_FLOW, FLOW, 1_550_011),
     ("packed", fpxgen.RECIPE_PACKED, DEST, 1_520_129),
-], ids=["mix", "flow", "packed"])
+    ("threshold", fpxgen.RECIPE_MIX, DEST, 1_515_520),
+    ("below", fpxgen.RECIPE_MIX, DEST, 1_515_519),
+    ("mix_big", fpxgen.RECIPE_MIX, DEST, 4_000_037),
+    ("flow_big", fpxgen.RECIPE_FLOW, FLOW, 3_500_017),
+], ids=["mix", "flow", "packed", "threshold", "below", "mix_big", "flow_big"])
 def test_dynamic_tail_parity(fpx, name, recipe, mode, n):
     p = fpxgen.Params(seed=0x5EED0100 + recipe, n_records=n, n_sites=3_000, recipe=recipe, p_fp64=0.5)
     hdr, arena = fpxgen.generate_host(p)
