@@ -597,11 +597,12 @@ def main():
         ents = merged[0][0]
 
     # e2e: the same metric through the public API with host buffers: per step,
-    # H2D of the step's inputs from pinned memory, scan, fetch (D2H of entries)
+    # H2D of the step's inputs from pinned memory, scan, fetch (D2H of entries).
+    # N > 1: every rank copies and scans its own shard, the step ends with the
+    # merged table on rank 0 in host memory (shared table: rank 0's fetch;
+    # NCCL merge: the merged arrays copied to the host); time = max over ranks.
     e2e = None
-    if world > 1:
-        e2e = {"value": None, "unit": UNIT, "reason": "e2e (host buffers) is measured at N = 1 only"}
-    if not args.no_e2e and world == 1:
+    if not args.no_e2e:
         try:
             wl.make_host_copies()
             torch.cuda.synchronize()
@@ -610,17 +611,36 @@ def main():
             tot = 0.0
             for i in range(args.e2e_steps + 1):
                 torch.cuda.synchronize()
+                if world > 1:
+                    dist.barrier()
                 e_a.record(stream)
                 h2d = wl.h2d()
-                h.reset(stream=stream)
+                if shared is not None:
+                    shared.reset(stream=stream)
+                else:
+                    h.reset(stream=stream)
                 wl.scan(h, stream)
-                got = h.fetch()  # synchronises; D2H of the entries
+                if shared is not None:
+                    shared.finish(stream=stream)
+                    got_bytes = h.fetch().nbytes if rank == 0 else 0  # synchronises; D2H of the entries
+                elif world > 1:
+                    k, c, f = fdist.merge_handle(h, stream=stream)
+                    got_bytes = sum(t.cpu().numel() * 8 for t in (k, c, f)) if rank == 0 else 0
+                else:
+                    got_bytes = h.fetch().nbytes
                 e_b.record(stream)
                 torch.cuda.synchronize()
                 if i > 0:  # first pass = warm-up
                     tot += e_a.elapsed_time(e_b)
-                d2h = got.nbytes
-            e2e = {"value": wl.lane_values / (tot / args.e2e_steps / 1e3), "unit": UNIT,
+                d2h = got_bytes
+            if world > 1:
+                tdev = torch.device("cpu") if dist.get_backend() == "gloo" else dev
+                t = torch.tensor([tot, float(h2d), float(d2h)], dtype=torch.float64, device=tdev)
+                tmax = t[:1].clone()
+                dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+                dist.all_reduce(t, op=dist.ReduceOp.SUM)
+                tot, h2d, d2h = float(tmax[0]), int(t[1]), int(t[2])
+            e2e = {"value": world * wl.lane_values / (tot / args.e2e_steps / 1e3), "unit": UNIT,
                    "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "steps": args.e2e_steps}
             wl.drop_host_copies()
         except Exception as ex:  # pragma: no cover - reported, not hidden

@@ -66,10 +66,13 @@ def test_two_ranks_on_one_gpu(merge):
     IPC mapping or falls back to the merge, saying so)."""
     lines = run(["-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2", "--master-addr=127.0.0.1",
                  f"--master-port={free_port()}", "bench.py", "--gpus", "2", "--debug-one-gpu", "--config", "c1",
-                 "--steps", "3", "--warmup", "3", "--no-e2e", "--merge", merge])
+                 "--steps", "3", "--warmup", "3", "--merge", merge])
     assert len(lines) == 1
     d = lines[0]
     assert d["n_gpus"] == 2 and len(d["per_rank"]["step_ms"]) == 2 and len(d["per_rank"]["scan_kernel_ms"]) == 2
     assert d["ms_per_step"] == pytest.approx(max(d["per_rank"]["step_ms"]), rel=1e-3)
     assert d["config"]["fetch_status"] == 0 and d["config"]["table_entries"] > 0
     assert d["cpu_baseline"] is None
+    # e2e at N = 2: both shards copied from host memory, merged table read back on rank 0
+    assert d["e2e"]["value"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
+    assert d["e2e"]["h2d_bytes_per_step"] >= 2 * d["config"]["algorithmic_bytes_per_gpu_step"]
