@@ -152,3 +152,27 @@ def test_report_detail_states():
     lines = report.analyzer_lines(e)
     assert lines[0].startswith("#GPU-FPX-ANA PROPAGATION: INF from source 1")
     assert lines[1].startswith("#GPU-FPX-ANA COMPARISON/DISAPPEARANCE: NaN from source 0")
+
+
+def test_header_is_plain_c_and_links(tmp_path):
+    """include/fpx.h is a C header: a C99 program (-pedantic, warnings as
+    errors) includes it, links libfpx.so and calls an entry point that needs
+    no GPU."""
+    import shutil
+
+    if shutil.which("gcc") is None:
+        pytest.skip("no gcc")
+    libdir = os.path.dirname(LIB)
+    src = tmp_path / "t.c"
+    src.write_text('#include "fpx.h"\n#include <stdio.h>\n'
+                   "int main(void) {\n  fpx_handle h = 0;\n  fpx_options o = {0, 0, 0};\n"
+                   "  fpx_rec_hdr r = {1u, 0xFFFFFFFFu, 0u, 0u};\n  (void)h; (void)o; (void)r;\n"
+                   '  printf("%s|%s\\n", fpx_strerror(FPX_OK), fpx_strerror(FPX_ERR_TABLE_FULL));\n'
+                   "  return (int)sizeof(fpx_entry) - 24;\n}\n")
+    exe = tmp_path / "t"
+    subprocess.run(["gcc", "-std=c99", "-Wall", "-Wextra", "-pedantic", "-Werror", "-I", os.path.dirname(HEADER),
+                    str(src), "-L", libdir, "-lfpx", f"-Wl,-rpath,{libdir}", "-o", str(exe)], check=True)
+    out = subprocess.run([str(exe)], capture_output=True, text=True)
+    assert out.returncode == 0, out.stderr
+    a, b = out.stdout.strip().split("|")
+    assert a and b and a != b
