@@ -12,6 +12,7 @@ import re
 import subprocess
 
 import numpy as np
+import pytest
 
 import fpxgen
 import oracle
