@@ -385,12 +385,14 @@ def test_reset_clears_every_key(fpx, newlog_capacity):
 
 
 @pytest.mark.parametrize("mode", [DEST, FLOW, FLOW_DETAIL])
-def test_irregular_layouts(fpx, mode):
+@pytest.mark.parametrize("n", [40_000, 1_700_003], ids=["static", "dynamic"])
+def test_irregular_layouts(fpx, mode, n):
     """Producer layouts the generator never makes: records in shuffled arena
     order, several records sharing planes (broadcast immediates),
     records whose planes run past the arena (bad), DEST scans of records with
-    sources (needed planes stop before the footprint ends)."""
-    p = fpxgen.Params(seed=17, n_records=40_000, n_sites=300, recipe=fpxgen.RECIPE_FLOW, p_fp64=0.4)
+    sources (needed planes stop before the footprint ends); at a size that
+    only uses static ranges and at one in the dynamic-tail regime."""
+    p = fpxgen.Params(seed=17, n_records=n, n_sites=300, recipe=fpxgen.RECIPE_FLOW, p_fp64=0.4)
     hdr, arena = fpxgen.generate_host(p)
     _, w = fpxgen.plan_injections(p, 400, flow=True)
     fpxgen.apply_host(w, hdr, arena)
