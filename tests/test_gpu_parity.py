@@ -14,7 +14,7 @@ import fpxgen
 import oracle
 from _records import (
     BF16, DEST, FLOW, FLOW_DETAIL, FP16, FP32, FP64, NAN, NONE, OP_FADD, Trace, describe_diff, entries_equal,
-    expected_from_injections, load_worked_cases, np_class, table_dict,
+    expected_from_injections, load_worked_cases, table_dict,
 )
 
 pytestmark = pytest.mark.gpu

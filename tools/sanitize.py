@@ -5,7 +5,6 @@ heads / tails, fetch / FETCH_NEW / reset / merge paths."""
 import os
 import sys
 
-import numpy as np
 import torch
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
