@@ -461,17 +461,29 @@ def test_scan_tensors_one_launch(fpx):
     ("below", fpxgen.RECIPE_MIX, DEST, 1_515_519),
     ("mix_big", fpxgen.RECIPE_MIX, DEST, 4_000_037),
     ("flow_big", fpxgen.RECIPE_FLOW, FLOW, 3_500_017),
-], ids=["mix", "flow", "packed", "threshold", "below", "mix_big", "flow_big"])
+    ("flow_detail", fpxgen.RECIPE_FLOW, FLOW_DETAIL, 1_600_001),
+    ("mix_noagg", fpxgen.RECIPE_MIX, DEST, 1_700_011),
+], ids=["mix", "flow", "packed", "threshold", "below", "mix_big", "flow_big", "flow_detail", "mix_noagg"])
 def test_dynamic_tail_parity(fpx, name, recipe, mode, n):
     p = fpxgen.Params(seed=0x5EED0100 + recipe, n_records=n, n_sites=3_000, recipe=recipe, p_fp64=0.5)
     hdr, arena = fpxgen.generate_host(p)
     inj, w = fpxgen.plan_injections(p, 3_000, flow=(recipe == fpxgen.RECIPE_FLOW))
     fpxgen.apply_host(w, hdr, arena)
     base = 3 * 10**9
-    got, st, stats = gpu_scan(fpx, hdr, arena, base=base, mode=mode)
+    flags = fpx.OPT_NO_WARP_AGG if name.endswith("noagg") else 0
+    got, st, stats = gpu_scan(fpx, hdr, arena, base=base, mode=mode, flags=flags)
     assert st == fpx.OK and stats.bad_records == 0
     assert_same(got, oracle_scan(hdr, arena, base, mode).entries())
-    assert table_dict(got) == expected_from_injections(hdr, inj, base, mode)
+    if mode == FLOW_DETAIL:  # detail splits entries further; (site, fmt, flow, kind) sums match
+        merged = {}
+        for e in got:
+            k = (int(e["site"]), int(e["fmt"]), int(e["flow"]), int(e["kind"]))
+            c = merged.setdefault(k, [0, 2**64 - 1])
+            c[0] += int(e["count"])
+            c[1] = min(c[1], int(e["first_index"]))
+        assert merged == expected_from_injections(hdr, inj, base, FLOW)
+    else:
+        assert table_dict(got) == expected_from_injections(hdr, inj, base, mode)
 
 
 def test_dynamic_tail_relaunch_and_streams(fpx):
