@@ -464,14 +464,24 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     fence_proxy_async_smem();
     // list l = 2 * fmt + partial; lists of lower formats come first
     const uint32_t tot_f = tf + tp;  // packed per-format item totals (<= 128 each)
-    if (in_tile && ni != 0u) {
+    const bool writes = in_tile && ni != 0u;
+    uint32_t at = 0u;
+    if (writes) {
       const uint32_t below = ((tot_f << (32 - 8 * fmt)) * 0x01010101u) >> 24;  // byte sum of formats < fmt
-      const uint32_t at = (fmt == 0u ? 0u : below) + (part ? ((tf >> (8 * fmt)) & 0xFFu) : 0u) +
-                          (((part ? sp - cp : sf - cf) >> (8 * fmt)) & 0xFFu);
+      at = (fmt == 0u ? 0u : below) + (part ? ((tf >> (8 * fmt)) & 0xFFu) : 0u) +
+           (((part ? sp - cp : sf - cf) >> (8 * fmt)) & 0xFFu);
+      sm.items[s][at] = make_uint2(slot, mask);
+    }
+#ifndef FPX_ITEMS_PREDICATED
+    // records with several items (HMMA fragments, FLOW sources) are absent
+    // from many traces: one vote skips their writes
+    if (__any_sync(FULL, writes && ni > 1u))
+#endif
+    {
       const uint32_t step = fmt == FPX_FP64 ? 2u : 1u;
 #pragma unroll
-      for (uint32_t j = 0; j < 4; ++j)  // ni <= 4
-        if (j < ni) sm.items[s][at + j] = make_uint2(slot + j * step, mask);
+      for (uint32_t j = 1; j < 4; ++j)  // ni <= 4
+        if (writes && j < ni) sm.items[s][at + j] = make_uint2(slot + j * step, mask);
     }
     if (lane == 0) {
       m.k = k;
