@@ -389,6 +389,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   uint32_t claim = 0;
   if (sch.nchunks != 0u && lane == 0) claim = atomicAdd(sch.ctr, 1u);
   const uint32_t* __restrict__ lane_base = arena + lane;
+  const uint4* __restrict__ hdr_lane = hdr + lane;  // this lane's header of a tile = hdr_lane[tile start]
   const uint64_t policy = policy_evict_first();
   const uint32_t g = (uint32_t)lane >> 3, q = (uint32_t)lane & 7u;
 
@@ -416,7 +417,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   };
   next_range();
   uint4 h = make_uint4(0, 0, 0, 0);
-  if ((uint32_t)lane < rem) h = ld_stream4(hdr + cursor + lane);
+  if ((uint32_t)lane < rem) h = ld_stream4(hdr_lane + cursor);
 
   // Build tile `s` from the prefetched headers and issue its copies.
   auto produce = [&](int s) {
@@ -498,8 +499,9 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const uint32_t foot = in_tile ? foot_all : 0u;
     const uint32_t d = a - slot;
     const uint32_t dmin = __reduce_min_sync(FULL, foot != 0u ? d : 0xFFFFFFFFu);
+    // (dmin + total <= 2^32: the run's arena planes fit the 32-bit plane index)
     const bool one_run = __all_sync(FULL, foot == 0u || (c == foot && d == dmin)) &&
-                         (uint64_t)dmin + total <= 0x100000000ull;
+                         (total == 0u || dmin <= 0u - total);
     if (one_run) {
       if (lane == 0) {
         mbar_arrive_expect_tx(&sm.bar[s], total * 128u);
@@ -529,7 +531,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     rem -= k;
     next_range();
     h = make_uint4(0, 0, 0, 0);
-    if ((uint32_t)lane < rem) h = ld_stream4(hdr + cursor + lane);
+    if ((uint32_t)lane < rem) h = ld_stream4(hdr_lane + cursor);
   };
 
   uint32_t phase = 0;  // bit s = parity to wait for on stage s
