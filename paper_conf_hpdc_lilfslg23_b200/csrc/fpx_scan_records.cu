@@ -106,9 +106,11 @@ struct RingCfg {
 // list l = 2 * fmt + partial.
 constexpr int NLISTS = 8;
 
+// StageMeta::k bit 31: the tile holds a record that must take the exact path
+constexpr uint32_t kForceBit = 0x80000000u;
 struct StageMeta {
-  uint32_t k;      // records in the tile (0 = no tile)
-  uint32_t force;  // tile holds a record that must take the exact path
+  uint32_t k;      // records in the tile (0 = no tile) | kForceBit
+  uint32_t pad0;
   uint64_t gidx0;  // global index of the tile's first record
   uint32_t tf;     // packed per-format item counts, full-mask lists (byte = format)
   uint32_t tp;     // same, partial-mask lists
@@ -451,14 +453,18 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const uint32_t fits = __ballot_sync(FULL, inrange && incl_planes <= (uint32_t)PLANES);
     const uint32_t k = (uint32_t)__popc(fits);
     const bool in_tile = (uint32_t)lane < k;
-    const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
-    if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
+    // bad records and forced (DIV) records are rare: one vote finds both
+    uint32_t force_any = 0u;
+    if (__any_sync(FULL, in_tile && (!ok || force))) {
+      const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
+      if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
+      force_any = __ballot_sync(FULL, in_tile && force);
+    }
     const uint32_t my_planes = planes_of_items(c8);
     const uint32_t c = in_tile ? my_planes : 0u;
     const uint32_t slot = incl_planes - my_planes;
     const uint32_t tf = __shfl_sync(FULL, sf, k - 1), tp = __shfl_sync(FULL, sp, k - 1);
     const uint32_t total = planes_of_items(tf) + planes_of_items(tp);
-    const uint32_t force_any = __ballot_sync(FULL, in_tile && force);
     // the ring slot may still be read by the previous consume of this stage:
     // order those generic reads before the async-proxy writes below
     __syncwarp();
@@ -485,8 +491,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
         if (writes && j < ni) sm.items[s][at + j] = make_uint2(slot + j * step, mask);
     }
     if (lane == 0) {
-      m.k = k;
-      m.force = force_any;
+      m.k = k | (force_any != 0u ? kForceBit : 0u);
       m.gidx0 = base_index + cursor;
       m.tf = tf;
       m.tp = tp;
@@ -542,7 +547,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const int s = (int)(i % STAGES);
     produce((int)((i + STAGES - 1) % STAGES));
     const StageMeta& m = sm.meta[s];
-    if (m.k == 0u) {
+    const uint32_t mk = m.k;  // records in the tile | kForceBit
+    if (mk == 0u) {
 #ifdef FPX_WARP_TIMES
       if (lane == 0 && gw < kMaxWarpTimes) g_warp_t1[gw] = globaltimer_ns();
 #endif
@@ -579,8 +585,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       consume_list<FPX_BF16, false>(w, seg[6], seg[7], ia, pa, g, q);
       consume_list<FPX_BF16, true>(w, seg[7], seg[8], ia, pa, g, q);
     }
-    if (__any_sync(FULL, w.hit_wide() || (halves && w.hit_half())) || m.force)
-      exact_tile_hdr<MODE>(hdr + (m.gidx0 - base_index), m.k, arena_planes, lane_base, sm.planes[s] + lane, lane,
+    if (__any_sync(FULL, w.hit_wide() || (halves && w.hit_half())) || (mk & kForceBit) != 0u)
+      exact_tile_hdr<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane, lane,
                            m.gidx0, tv, [](uint32_t meta) {
                              bool f;
                              const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, f, f);
