@@ -460,11 +460,11 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
       force_any = __ballot_sync(FULL, in_tile && force);
     }
-    const uint32_t my_planes = planes_of_items(c8);
+    const uint32_t my_planes = ni << (fmt == FPX_FP64 ? 1u : 0u);  // = planes_of_items(c8)
     const uint32_t c = in_tile ? my_planes : 0u;
     const uint32_t slot = incl_planes - my_planes;
     const uint32_t tf = __shfl_sync(FULL, sf, k - 1), tp = __shfl_sync(FULL, sp, k - 1);
-    const uint32_t total = planes_of_items(tf) + planes_of_items(tp);
+    const uint32_t total = __shfl_sync(FULL, incl_planes, k - 1);  // the tile's planes
     // the ring slot may still be read by the previous consume of this stage:
     // order those generic reads before the async-proxy writes below
     __syncwarp();
