@@ -270,6 +270,18 @@ struct Witness {
   }
 };
 
+// Predicated streaming 128-bit global load (zeros when !p), without a branch.
+__device__ __forceinline__ uint4 ld_stream4_if(bool p, const void* ptr) {
+  uint4 v;
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %4, 0;\n\t"
+      "mov.u32 %0, 0;\n\tmov.u32 %1, 0;\n\tmov.u32 %2, 0;\n\tmov.u32 %3, 0;\n\t"
+      "@q ld.global.nc.L1::no_allocate.v4.u32 {%0, %1, %2, %3}, [%5];\n\t}"
+      : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+      : "r"((uint32_t)p), "l"(ptr));
+  return v;
+}
+
 // 128-bit shared load at a byte address.
 __device__ __forceinline__ uint4 lds128(uint32_t addr) {
   uint4 v;
@@ -408,7 +420,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   uint32_t rem = (uint32_t)(end - start);
   // at the end of a range: move into the claimed chunk and claim the next
   auto next_range = [&]() {
-    if (rem == 0u && sch.nchunks != 0u) {
+    if (rem == 0u) {
+      if (sch.nchunks == 0u) return;
       const uint32_t c = __shfl_sync(FULL, claim, 0);
       if (c < sch.nchunks) {
         cursor = c < sch.nbig ? sch.dyn0 + (uint64_t)c * sch.chunk : sch.dyn1 + (uint64_t)(c - sch.nbig) * TILE;
@@ -418,8 +431,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     }
   };
   next_range();
-  uint4 h = make_uint4(0, 0, 0, 0);
-  if ((uint32_t)lane < rem) h = ld_stream4(hdr_lane + cursor);
+  uint4 h = ld_stream4_if((uint32_t)lane < rem, hdr_lane + cursor);
 
   // Build tile `s` from the prefetched headers and issue its copies.
   auto produce = [&](int s) {
@@ -535,8 +547,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     cursor += k;
     rem -= k;
     next_range();
-    h = make_uint4(0, 0, 0, 0);
-    if ((uint32_t)lane < rem) h = ld_stream4(hdr_lane + cursor);
+    h = ld_stream4_if((uint32_t)lane < rem, hdr_lane + cursor);
   };
 
   uint32_t phase = 0;  // bit s = parity to wait for on stage s
