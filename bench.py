@@ -94,10 +94,10 @@ class ClockSampler:
         self.samples = []
         self._stop = threading.Event()
         self._t = None
+        self._one = None
 
-    def _run(self):
-        # NVML (what nvidia-smi reads) every 10 ms; nvidia-smi itself takes
-        # ~0.3 s per query, too slow for a sub-second timed region
+    def _nvml(self):
+        """NVML handle and a one-sample reader (None if NVML is unavailable)."""
         try:
             import pynvml
 
@@ -106,14 +106,27 @@ class ClockSampler:
             bits = (pynvml.nvmlClocksEventReasonHwSlowdown, pynvml.nvmlClocksEventReasonHwThermalSlowdown,
                     pynvml.nvmlClocksEventReasonSwThermalSlowdown, pynvml.nvmlClocksEventReasonSwPowerCap)
             mx = pynvml.nvmlDeviceGetMaxClockInfo(dev, pynvml.NVML_CLOCK_SM)
-            while not self._stop.is_set():
+
+            def one():
                 sm = pynvml.nvmlDeviceGetClockInfo(dev, pynvml.NVML_CLOCK_SM)
                 r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(dev)
                 self.samples.append([str(sm), str(mx), hex(r)] + ["Active" if r & b else "Not Active" for b in bits])
-                self._stop.wait(0.01)
-            return
+
+            one()  # fails here, before the timed region, if NVML cannot read this GPU
+            return one
         except Exception:
-            pass
+            return None
+
+    def _run(self):
+        # NVML (what nvidia-smi reads) every 10 ms; nvidia-smi itself takes
+        # ~0.3 s per query, too slow for a sub-second timed region
+        if self._one is not None:
+            while not self._stop.wait(0.01):
+                try:
+                    self._one()
+                except Exception:
+                    return
+            return
         while not self._stop.is_set():
             try:
                 out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
@@ -125,6 +138,7 @@ class ClockSampler:
             self._stop.wait(0.05)
 
     def __enter__(self):
+        self._one = self._nvml()  # NVML set up (and one sample taken) before the timed region starts
         self._t = threading.Thread(target=self._run, daemon=True)
         self._t.start()
         return self
@@ -132,6 +146,11 @@ class ClockSampler:
     def __exit__(self, *a):
         self._stop.set()
         self._t.join(timeout=10)
+        if self._one is not None:  # and one as it ends, so short regions hold two
+            try:
+                self._one()
+            except Exception:
+                pass
 
     def summary(self):
         if not self.samples:
