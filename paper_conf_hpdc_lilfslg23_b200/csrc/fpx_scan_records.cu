@@ -486,9 +486,12 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const bool writes = in_tile && ni != 0u;
     uint32_t at = 0u;
     if (writes) {
-      const uint32_t below = ((tot_f << (32 - 8 * fmt)) * 0x01010101u) >> 24;  // byte sum of formats < fmt
-      at = (fmt == 0u ? 0u : below) + (part ? ((tf >> (8 * fmt)) & 0xFFu) : 0u) +
-           (((part ? sp - cp : sf - cf) >> (8 * fmt)) & 0xFFu);
+      // byte f of `below`: items of the formats before f; byte f of `own`:
+      // this record's place among format f's items (full list first).  Every
+      // byte stays <= 40 (items <= planes), so the packed sums never carry.
+      const uint32_t below = (tot_f * 0x01010101u) << 8;
+      const uint32_t own = part ? tf + (sp - cp) : sf - cf;
+      at = ((below + own) >> (8 * fmt)) & 0xFFu;
       sm.items[s][at] = make_uint2(slot, mask);
     }
 #ifndef FPX_ITEMS_PREDICATED
