@@ -459,7 +459,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     scan_step<4>(sf), scan_step<4>(sp);
     scan_step<8>(sf), scan_step<8>(sp);
     scan_step<16>(sf), scan_step<16>(sp);
-    const uint32_t incl_planes = planes_of_items(sf) + planes_of_items(sp);
+    // a lane is in one of the two lists, so sf + sp stays <= 128 per byte
+    const uint32_t incl_planes = planes_of_items(sf + sp);
     // the tile = leading records whose planes fit the stage (>= 1 record);
     // incl_planes never decreases over the lanes, so `fits` is a lane prefix
     const uint32_t fits = __ballot_sync(FULL, inrange && incl_planes <= (uint32_t)PLANES);
