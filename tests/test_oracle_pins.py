@@ -17,8 +17,8 @@ import pytest
 import fpxgen
 import oracle
 from _records import (
-    BF16, DEST, DIV0, FLOW, FLOW_DETAIL, FP16, FP32, FP64, GEN, INF, KILL, NAN, NONE, OP_DIV, OP_FADD, OP_FFMA,
-    OP_FMNMX, OP_FMUL, OP_FSEL, OP_FSETP, OP_RCP, OP_RCP64H, PROP, SUB, Trace, expected_from_injections,
+    BF16, DEST, DIV0, FLOW, FLOW_DETAIL, FP16, FP32, FP64, GEN, INF, KILL, NAN, NONE, OP_DIV, OP_DSETP, OP_FADD,
+    OP_FFMA, OP_FMNMX, OP_FMUL, OP_FSEL, OP_FSET, OP_FSETP, OP_RCP, OP_RCP64H, PROP, SUB, Trace, expected_from_injections,
     load_worked_cases, np_class, table_dict, words_of,
 )
 
@@ -141,9 +141,9 @@ def _ieee_expect(fmt, op, dest, srcs):
     cls = lambda v: int(np_class(fmt, np.array([_bits(fmt, v)], dtype=np.uint64))[0])
     kind = {C_NAN: NAN, C_INF: INF, C_SUB: SUB}
     D = None
-    if dest is not None:
+    if dest is not None and op != OP_FSET:  # FSET's destination is an integer mask (R10)
         cd = cls(dest)
-        if op == OP_RCP:
+        if op in (OP_RCP, OP_RCP64H):
             D = DIV0 if cd in (C_NAN, C_INF) else None
         elif op == OP_DIV and srcs[1] == 0 and np.isfinite(srcs[0]) and srcs[0] != 0:
             D = DIV0
@@ -166,7 +166,7 @@ def _ieee_expect(fmt, op, dest, srcs):
     if S is not None:
         classes = [cls(s) for s in srcs]
         det = 1 + next(i for i, c in enumerate(classes) if sev[c] == max(sev[x] for x in classes))
-        if op in (OP_FSEL, OP_FSETP, OP_FMNMX):
+        if op in (OP_FSEL, OP_FSET, OP_FSETP, OP_FMNMX, OP_DSETP):  # Table 1's right column
             det |= 4
     return (None if D is None else (D, NONE)), fl, det
 
@@ -181,7 +181,12 @@ def _brute_records(fmt):
             cases.append((OP_FMUL, a * b, [a, b]))
             cases.append((OP_DIV, a / b, [a, b]))
             cases.append((OP_FMNMX, np.fmin(a, b), [a, b]))  # IEEE-2008 minNum
-            cases.append((OP_FSETP, None, [a, b]))
+            # compare-and-set predicate (FSETP / DSETP, T1 P:101-110): no FP destination
+            cases.append((OP_FSETP if fmt == FP32 else OP_DSETP, None, [a, b]))
+            if fmt == FP32:
+                # FSET (T1: FP32 Compare And Set) writes the integer mask of a < b:
+                # 0xFFFFFFFF when true -- a NaN bit pattern that is not a NaN (R10)
+                cases.append((OP_FSET, np.array([0xFFFFFFFF if a < b else 0], np.uint32).view(np.float32)[0], [a, b]))
             cases.append((OP_FSEL, a, [a, b]))  # predicate true: selects a
             cases.append((OP_FSEL, b, [a, b]))  # predicate false: selects b
         for a, b, c in itertools.product(sp, sp, sp):
@@ -197,13 +202,13 @@ def test_bruteforce_ieee_ops(fmt):
     through real IEEE ops; each record scanned alone so its (kind, flow) is
     checked against numpy's classification of the real result."""
     cases = _brute_records(fmt)
-    opmap = {OP_FADD: OP_FADD, OP_FMUL: OP_FMUL, OP_DIV: OP_DIV, OP_FMNMX: OP_FMNMX, OP_FSETP: OP_FSETP,
-             OP_FSEL: OP_FSEL, OP_FFMA: OP_FFMA, OP_RCP: OP_RCP}
-    if fmt == FP64:
-        opmap[OP_RCP] = OP_RCP64H
+    rcp = OP_RCP if fmt == FP32 else OP_RCP64H
+    ops_seen = set()
     for op, dest, srcs in cases:
+        op = rcp if op == OP_RCP else op
+        ops_seen.add(op)
         tr = Trace()
-        tr.add_value_record(9, opmap[op], fmt, 0xFFFFFFFF, None if dest is None else _bits(fmt, dest),
+        tr.add_value_record(9, op, fmt, 0xFFFFFFFF, None if dest is None else _bits(fmt, dest),
                             [_bits(fmt, s) for s in srcs])
         hdr, arena = tr.arrays()
         exp_d, exp_f, exp_det = _ieee_expect(fmt, op, dest, srcs)
@@ -217,6 +222,8 @@ def test_bruteforce_ieee_ops(fmt):
             if got is not None:
                 assert int(ents[0]["count"]) == 32
                 assert int(ents[0]["detail"]) == (exp_det if mode == FLOW_DETAIL else 0), (op, srcs, ents)
+    assert ops_seen == ({OP_FADD, OP_FMUL, OP_DIV, OP_FMNMX, OP_FSETP, OP_FSET, OP_FSEL, OP_FFMA, OP_RCP} if fmt == FP32
+                        else {OP_FADD, OP_FMUL, OP_DIV, OP_FMNMX, OP_DSETP, OP_FSEL, OP_FFMA, OP_RCP64H})
 
 
 # --------------------------------------------------------------------------
@@ -389,3 +396,66 @@ def test_tensor_scan_vs_numpy():
 def test_key_layout():
     assert oracle.key(0x12345678, FP64, PROP, DIV0) == (0x12345678 << 32) | (1 << 4) | (2 << 2) | 3
     assert words_of(FP64, 0x7FF0000000000001) == [1, 0x7FF00000]
+
+
+# --------------------------------------------------------------------------
+# R19: a recorded division on packed FP16x2 / BF16x2 words is checked per
+# half, each half with the dividend / divisor halves at the same position;
+# pinned against real half-precision IEEE division (numpy float16, torch
+# bfloat16 on the CPU) and numpy's classification of the real quotient.
+# --------------------------------------------------------------------------
+_HALF_SPECIALS = {
+    FP16: [0x0000, 0x8000, 0x3E00, 0x0123, 0x7C00, 0xFC00, 0x7E00],  # +0 -0 1.5 SUB +INF -INF NaN
+    BF16: [0x0000, 0x8000, 0x3FC0, 0x0012, 0x7F80, 0xFF80, 0x7FC0],
+}
+
+
+def _half_div(fmt, a, b):
+    """IEEE quotient of two halves (bit patterns) in the half format itself."""
+    if fmt == FP16:
+        x = np.array([a, b], np.uint16).view(np.float16)
+        with np.errstate(all="ignore"):
+            return int(np.array([x[0] / x[1]], np.float16).view(np.uint16)[0])
+    import torch
+
+    x = torch.tensor([a, b], dtype=torch.int32).to(torch.int16).view(torch.bfloat16)
+    return int((x[0:1] / x[1:2]).view(torch.int16).to(torch.int32)[0]) & 0xFFFF
+
+
+@pytest.mark.parametrize("fmt", [FP16, BF16])
+def test_div_packed_halves_vs_ieee(fmt):
+    sp = _HALF_SPECIALS[fmt]
+    combos = list(itertools.product(sp, sp))
+    tr = Trace(seed=19)
+    exp = {}
+    for i, (a0, b0) in enumerate(combos):
+        a1, b1 = combos[(7 * i + 3) % len(combos)]
+        q0, q1 = _half_div(fmt, a0, b0), _half_div(fmt, a1, b1)
+        tr.add(i, OP_DIV, fmt, 0xFFFFFFFF, [q0 | (q1 << 16)], [[a0 | (a1 << 16)], [b0 | (b1 << 16)]])
+        for a, b, q in ((a0, b0, q0), (a1, b1, q1)):
+            fa = np_class(fmt, np.array([a], np.uint64))[0]
+            a_finite_nonzero = fa in (C_SUB, CLEAN) and (a & 0x7FFF) != 0
+            if (b & 0x7FFF) == 0 and a_finite_nonzero:  # IEEE divideByZero (R1)
+                k = DIV0
+            else:
+                k = {C_NAN: NAN, C_INF: INF, C_SUB: SUB}.get(int(np_class(fmt, np.array([q], np.uint64))[0]))
+            if k is not None:
+                e = exp.setdefault((i, fmt, NONE, k), [0, i])
+                e[0] += 32
+    hdr, arena = tr.arrays()
+    t = oracle.Table()
+    t.scan_records(hdr, arena, mode=DEST)
+    assert t.bad_records == 0
+    got = table_dict(t.entries())
+    assert got == exp
+    assert {k[3] for k in exp} == {NAN, INF, SUB, DIV0}  # every kind occurs
+    # R19: with a multi-word destination (dwords != source width) the rule
+    # falls back to the destination class: 1/0 = INF reports INF, not DIV0
+    tr = Trace()
+    one = 0x3C00 if fmt == FP16 else 0x3F80
+    inf = 0x7C00 if fmt == FP16 else 0x7F80
+    tr.add(1, OP_DIV, fmt, 0x1, [inf | (one << 16), one | (one << 16)], [[one | (one << 16)], [0]])
+    h, a = tr.arrays()
+    t = oracle.Table()
+    t.scan_records(h, a)
+    assert table_dict(t.entries()) == {(1, fmt, NONE, INF): [1, 0]}
