@@ -515,8 +515,9 @@ def main():
                     help="ablation: per-lane table updates in the exact path (FPX_OPT_NO_WARP_AGG)")
     ap.add_argument("--debug-one-gpu", action="store_true",
                     help="testing only: every rank on cuda:0 with gloo (exercises the N > 1 code paths on one GPU)")
-    ap.add_argument("--merge", default="peer", choices=["nccl", "peer"],
-                    help="N > 1: NCCL merge of per-GPU tables, or one shared table updated over NVLink peer memory")
+    ap.add_argument("--merge", default="nccl", choices=["nccl", "peer"],
+                    help="N > 1: NCCL merge of per-GPU tables (default; SURVEY §8 e), or one shared table updated "
+                         "over NVLink peer memory with system-scope atomics (not yet run across distinct GPUs)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     cfg = dict(CONFIGS[args.config])

@@ -259,9 +259,13 @@ fpx_status fpx_scan_tensors(fpx_handle h, const fpx_tensor_desc* descs, uint32_t
  * caller-allocated host memory.  flags = FPX_FETCH_ALL: every entry;
  * FPX_FETCH_NEW: only keys first inserted since the previous FETCH_NEW call
  * (the paper's "only push new combinations", served from the device
- * new-key log).  *n_total receives the number of entries available.  If
- * capacity < *n_total the first `capacity` are written and FPX_ERR_TRUNCATED
- * is returned; otherwise the sticky device status (FPX_ERR_TABLE_FULL before
+ * new-key log).  *n_total receives the number of entries available (FETCH_NEW:
+ * the number of new keys not yet returned).  If capacity < *n_total the first
+ * `capacity` are written and FPX_ERR_TRUNCATED is returned — FETCH_ALL: the
+ * first in key order; FETCH_NEW: the first `capacity` new keys in insertion
+ * order (sorted by key among themselves), and only those count as returned,
+ * so the next FETCH_NEW call continues with the rest (capacity 0 only
+ * queries).  Otherwise the sticky device status (FPX_ERR_TABLE_FULL before
  * FPX_ERR_BAD_RECORD) or FPX_OK.  host_out may be NULL when capacity == 0. */
 fpx_status fpx_table_fetch(fpx_handle h, fpx_entry* host_out, uint64_t capacity,
                            uint64_t* n_total, uint32_t flags);

@@ -38,7 +38,8 @@ struct fpx_ctx {
   ListEntry* d_list = nullptr;
   ListEntry* h_list = nullptr;
   uint32_t list_cap = 0;
-  cudaEvent_t list_copied = nullptr;
+  cudaEvent_t list_copied = nullptr;  // the last H2D copy out of h_list is done
+  cudaEvent_t list_used = nullptr;    // the last launch reading d_list is done
   // record-scan chunk counters (fpx_scan_records.cu Sched): kSchedSlots
   // pairs, one per launch in turn, so that launches in flight on different
   // streams never share one
@@ -93,27 +94,45 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) ==
 
 fpx_status ensure_scratch(fpx_ctx* h) {
   if (h->d_keys) return FPX_OK;
+  // allocate into locals and commit only when every allocation succeeded, so
+  // a failure leaves the handle without scratch (the next call retries)
+  // instead of with a half-built set
   const size_t b = sizeof(uint64_t) * h->slots;
-  CK(cudaMalloc(&h->d_keys, b));
-  CK(cudaMalloc(&h->d_counts, b));
-  CK(cudaMalloc(&h->d_first, b));
-  CK(cudaMalloc(&h->d_keys2, b));
-  CK(cudaMalloc(&h->d_idx, b));
-  CK(cudaMalloc(&h->d_idx2, b));
-  CK(cudaMalloc(&h->d_n, sizeof(unsigned long long)));
+  void* p[7] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+  void* temp = nullptr;
   size_t t1 = 0, t2 = 0;
-  CK(sort_keys_with_index(nullptr, &t1, h->d_keys, h->d_keys2, h->d_idx, h->d_idx2, h->slots, nullptr));
-  CK(unique_keys(nullptr, &t2, h->d_keys, h->d_keys2, h->d_n, h->slots, nullptr));
+  cudaError_t e = cudaSuccess;
+  for (int i = 0; i < 7 && e == cudaSuccess; ++i) e = cudaMalloc(&p[i], i < 6 ? b : sizeof(unsigned long long));
+  if (e == cudaSuccess)
+    e = sort_keys_with_index(nullptr, &t1, static_cast<uint64_t*>(p[0]), static_cast<uint64_t*>(p[3]),
+                             static_cast<uint64_t*>(p[4]), static_cast<uint64_t*>(p[5]), h->slots, nullptr);
+  if (e == cudaSuccess)
+    e = unique_keys(nullptr, &t2, static_cast<uint64_t*>(p[0]), static_cast<uint64_t*>(p[3]),
+                    static_cast<unsigned long long*>(p[6]), h->slots, nullptr);
+  if (e == cudaSuccess) e = cudaMalloc(&temp, std::max(t1, t2));
+  if (e != cudaSuccess) {
+    for (void* q : p)
+      if (q) cudaFree(q);
+    return cuda_err(e, "ensure_scratch");
+  }
+  h->d_keys = static_cast<uint64_t*>(p[0]);
+  h->d_counts = static_cast<uint64_t*>(p[1]);
+  h->d_first = static_cast<uint64_t*>(p[2]);
+  h->d_keys2 = static_cast<uint64_t*>(p[3]);
+  h->d_idx = static_cast<uint64_t*>(p[4]);
+  h->d_idx2 = static_cast<uint64_t*>(p[5]);
+  h->d_n = static_cast<unsigned long long*>(p[6]);
+  h->d_temp = temp;
   h->temp_bytes = std::max(t1, t2);
-  CK(cudaMalloc(&h->d_temp, h->temp_bytes));
   return FPX_OK;
 }
 
 fpx_status ensure_temp(fpx_ctx* h, size_t need) {
   if (need <= h->temp_bytes) return FPX_OK;
-  if (h->d_temp) CK(cudaFree(h->d_temp));
-  h->d_temp = nullptr;
-  CK(cudaMalloc(&h->d_temp, need));
+  void* t = nullptr;
+  CK(cudaMalloc(&t, need));
+  if (h->d_temp) cudaFree(h->d_temp);
+  h->d_temp = t;
   h->temp_bytes = need;
   return FPX_OK;
 }
@@ -196,39 +215,31 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   if (!h) return FPX_ERR_NOMEM;
   h->device = device;
   h->variant = (o.flags & FPX_OPT_SCAN_LDG) ? 1u : 0u;
-  CK(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, device));
   h->slots = 1ull << o.table_log2_slots;
+  // every failure below releases what was built so far through fpx_close
+  // (which tolerates the members still null)
+  auto fail = [&](fpx_status st) {
+    cudaGetLastError();
+    fpx_close(h);
+    return st;
+  };
+  cudaError_t e = cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, device);
+  if (e != cudaSuccess) return fail(cuda_err(e, "cudaDeviceGetAttribute"));
   // the log never holds more keys than the table has slots
   const uint64_t cap = o.newlog_capacity ? std::min<uint64_t>(o.newlog_capacity, h->slots) : h->slots;
-  Slot* slots = nullptr;
-  unsigned long long* log = nullptr;
-  unsigned int* log_slot = nullptr;
-  Ctl* ctl = nullptr;
-  if (cudaMalloc(&slots, sizeof(Slot) * h->slots) != cudaSuccess ||
-      cudaMalloc(&log, sizeof(unsigned long long) * cap) != cudaSuccess ||
-      cudaMalloc(&log_slot, sizeof(unsigned int) * cap) != cudaSuccess ||
-      cudaMalloc(&ctl, sizeof(Ctl)) != cudaSuccess || cudaMallocHost(&h->h_ctl, sizeof(Ctl)) != cudaSuccess) {
-    cudaGetLastError();
-    if (slots) cudaFree(slots);
-    if (log) cudaFree(log);
-    if (log_slot) cudaFree(log_slot);
-    if (ctl) cudaFree(ctl);
-    delete h;
-    return FPX_ERR_NOMEM;
-  }
-  h->tv.slots = slots;
+  if (cudaMalloc(&h->tv.slots, sizeof(Slot) * h->slots) != cudaSuccess ||
+      cudaMalloc(&h->tv.newlog, sizeof(unsigned long long) * cap) != cudaSuccess ||
+      cudaMalloc(&h->tv.newlog_slot, sizeof(unsigned int) * cap) != cudaSuccess ||
+      cudaMalloc(&h->tv.ctl, sizeof(Ctl)) != cudaSuccess || cudaMallocHost(&h->h_ctl, sizeof(Ctl)) != cudaSuccess)
+    return fail(FPX_ERR_NOMEM);
   h->tv.mask = h->slots - 1;
-  h->tv.newlog = log;
-  h->tv.newlog_slot = log_slot;
   h->tv.newlog_cap = cap;
-  h->tv.ctl = ctl;
   h->tv.flags = o.flags & FPX_OPT_NO_WARP_AGG;
-  CK(launch_table_reset(h->tv, h->slots, nullptr));
-  if (!alloc_sched(h)) {
-    fpx_close(h);
-    return FPX_ERR_NOMEM;
-  }
-  CK(cudaStreamSynchronize(nullptr));
+  e = launch_table_reset(h->tv, h->slots, nullptr);
+  if (e != cudaSuccess) return fail(cuda_err(e, "launch_table_reset"));
+  if (!alloc_sched(h)) return fail(FPX_ERR_NOMEM);
+  e = cudaStreamSynchronize(nullptr);
+  if (e != cudaSuccess) return fail(cuda_err(e, "cudaStreamSynchronize"));
   *out = h;
   return FPX_OK;
 }
@@ -284,10 +295,11 @@ fpx_status fpx_scan_tensors(fpx_handle h, const fpx_tensor_desc* descs, uint32_t
   if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   if (!h->list_copied) CK(cudaEventCreateWithFlags(&h->list_copied, cudaEventDisableTiming));
-  CK(cudaEventSynchronize(h->list_copied));  // the staging buffer's previous copy is done
+  if (!h->list_used) CK(cudaEventCreateWithFlags(&h->list_used, cudaEventDisableTiming));
+  CK(cudaEventSynchronize(h->list_copied));  // the host staging buffer's previous copy is done
   if (m > h->list_cap) {
     if (h->d_list) {
-      CK(cudaStreamSynchronize(h->last_stream));  // earlier launches may still read the old table
+      CK(cudaEventSynchronize(h->list_used));  // the launch reading the old table (any stream) is done
       CK(cudaFree(h->d_list));
     }
     if (h->h_list) CK(cudaFreeHost(h->h_list));
@@ -298,6 +310,9 @@ fpx_status fpx_scan_tensors(fpx_handle h, const fpx_tensor_desc* descs, uint32_t
     if (cudaMalloc(&h->d_list, sizeof(ListEntry) * cap) != cudaSuccess ||
         cudaMallocHost(&h->h_list, sizeof(ListEntry) * cap) != cudaSuccess) {
       cudaGetLastError();
+      if (h->d_list) cudaFree(h->d_list);
+      h->d_list = nullptr;
+      h->h_list = nullptr;
       h->list_cap = 0;
       return FPX_ERR_NOMEM;
     }
@@ -328,9 +343,13 @@ fpx_status fpx_scan_tensors(fpx_handle h, const fpx_tensor_desc* descs, uint32_t
     vsum += nvec;
     ssum += head + tail;
   }
+  // the device table may still be read by the previous launch on another
+  // stream: this stream waits for it before overwriting
+  CK(cudaStreamWaitEvent(s, h->list_used, 0));
   CK(cudaMemcpyAsync(h->d_list, h->h_list, sizeof(ListEntry) * m, cudaMemcpyHostToDevice, s));
   CK(cudaEventRecord(h->list_copied, s));
   CK(launch_scan_tensor_list(h->d_list, m, vsum, ssum, h->tv, h->num_sms, s));
+  CK(cudaEventRecord(h->list_used, s));
   h->last_stream = s;
   return FPX_OK;
 }
@@ -344,20 +363,26 @@ fpx_status fpx_table_fetch(fpx_handle h, fpx_entry* host_out, uint64_t capacity,
   CK(cudaStreamSynchronize(s));
   fpx_status st = ensure_scratch(h);
   if (st != FPX_OK) return st;
-  uint64_t n = 0;
+  uint64_t n = 0, new_total = 0;
   if (flags == FPX_FETCH_ALL) {
     st = sorted_entries(h, s, nullptr, 0, &n);
+    new_total = n;
   } else {
-    // keys inserted since the previous FETCH_NEW, read from the device log
+    // keys inserted since the previous FETCH_NEW, read from the device log in
+    // insertion order: a window of at most `capacity` of them (sorted by key
+    // within it), and the cursor moves past exactly the keys returned, so a
+    // truncated call loses nothing (the next call continues from there)
     CK(cudaMemcpyAsync(h->h_ctl, h->tv.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     const uint64_t tail = std::min<uint64_t>(h->h_ctl->newlog_tail, h->tv.newlog_cap);
     const uint64_t from = std::min<uint64_t>(h->newlog_cursor, tail);
-    st = sorted_entries(h, s, reinterpret_cast<const uint64_t*>(h->tv.newlog) + from, tail - from, &n);
-    if (st == FPX_OK) h->newlog_cursor = tail;
+    new_total = tail - from;
+    const uint64_t take = std::min<uint64_t>(new_total, capacity);
+    st = sorted_entries(h, s, reinterpret_cast<const uint64_t*>(h->tv.newlog) + from, take, &n);
+    if (st == FPX_OK) h->newlog_cursor = from + take;
   }
   if (st != FPX_OK) return st;
-  *n_total = n;
+  *n_total = new_total;
   const uint64_t m = std::min(n, capacity);
   if (m) {
     std::vector<uint64_t> k(m), c(m), f(m);
@@ -378,7 +403,7 @@ fpx_status fpx_table_fetch(fpx_handle h, fpx_entry* host_out, uint64_t capacity,
       host_out[i] = e;
     }
   }
-  if (capacity < n) return FPX_ERR_TRUNCATED;
+  if (capacity < new_total) return FPX_ERR_TRUNCATED;
   return sticky_status(h, s);
 }
 
@@ -500,6 +525,9 @@ fpx_status fpx_table_export(fpx_handle h, fpx_ipc_table* out) {
   out->newlog_capacity = (uint32_t)h->tv.newlog_cap;
   out->home_device = h->device;
   out->magic = FPX_IPC_MAGIC;
+  // other GPUs will update this table concurrently: the home's own scans
+  // switch to system-scope atomics too
+  h->tv.flags |= TV_SHARED;
   return FPX_OK;
 }
 
@@ -516,7 +544,11 @@ fpx_status fpx_open_attached(int device, const fpx_ipc_table* t, fpx_handle* out
   if (!h) return FPX_ERR_NOMEM;
   h->device = device;
   h->attached = true;
-  CK(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, device));
+  cudaError_t ea = cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, device);
+  if (ea != cudaSuccess) {
+    delete h;
+    return cuda_err(ea, "cudaDeviceGetAttribute");
+  }
   h->slots = 1ull << t->table_log2_slots;
   void* ptrs[4] = {nullptr, nullptr, nullptr, nullptr};
   for (int i = 0; i < 4; ++i) {
@@ -535,6 +567,7 @@ fpx_status fpx_open_attached(int device, const fpx_ipc_table* t, fpx_handle* out
   h->tv.newlog_slot = static_cast<unsigned int*>(ptrs[2]);
   h->tv.ctl = static_cast<Ctl*>(ptrs[3]);
   h->tv.newlog_cap = t->newlog_capacity;
+  h->tv.flags = TV_SHARED;  // concurrent updates from several GPUs: system-scope atomics
   if (cudaMallocHost(&h->h_ctl, sizeof(Ctl)) != cudaSuccess) {
     for (int j = 0; j < 4; ++j) cudaIpcCloseMemHandle(ptrs[j]);
     delete h;
@@ -544,7 +577,11 @@ fpx_status fpx_open_attached(int device, const fpx_ipc_table* t, fpx_handle* out
     fpx_close(h);
     return FPX_ERR_NOMEM;
   }
-  CK(cudaStreamSynchronize(nullptr));
+  ea = cudaStreamSynchronize(nullptr);
+  if (ea != cudaSuccess) {
+    fpx_close(h);
+    return cuda_err(ea, "cudaStreamSynchronize");
+  }
   *out = h;
   return FPX_OK;
 }
@@ -569,6 +606,7 @@ fpx_status fpx_close(fpx_handle h) {
     if (h->h_list) cudaFreeHost(h->h_list);
     if (h->d_list) cudaFree(h->d_list);
     if (h->list_copied) cudaEventDestroy(h->list_copied);
+    if (h->list_used) cudaEventDestroy(h->list_used);
     for (void* p : {(void*)h->d_keys, (void*)h->d_counts, (void*)h->d_first, (void*)h->d_keys2, (void*)h->d_idx,
                     (void*)h->d_idx2, (void*)h->d_n, h->d_temp, (void*)h->d_sched})
       if (p) cudaFree(p);

@@ -104,6 +104,23 @@ __device__ __forceinline__ unsigned long long hash_key(unsigned long long k) {
   return k;
 }
 
+// Atomics on the table and its counters.  The CUDA memory model makes an
+// atomic indivisible only among the threads of its scope: a table shared with
+// other GPUs (TV_SHARED: the home handle after fpx_table_export, every
+// fpx_open_attached handle) is updated from several devices at once over
+// NVLink, so its atomics are system-scope; a local table keeps device scope.
+__device__ __forceinline__ unsigned long long t_cas(const TableView& tv, unsigned long long* a, unsigned long long c,
+                                                    unsigned long long v) {
+  return (tv.flags & TV_SHARED) ? atomicCAS_system(a, c, v) : atomicCAS(a, c, v);
+}
+__device__ __forceinline__ unsigned long long t_add(const TableView& tv, unsigned long long* a, unsigned long long v) {
+  return (tv.flags & TV_SHARED) ? atomicAdd_system(a, v) : atomicAdd(a, v);
+}
+__device__ __forceinline__ void t_min(const TableView& tv, unsigned long long* a, unsigned long long v) {
+  if (tv.flags & TV_SHARED) atomicMin_system(a, v);
+  else atomicMin(a, v);
+}
+
 // Insert-or-update.  Linear probing over the whole table: an event is only
 // dropped (and TABLE_FULL raised) when every slot holds another key.
 static __device__ __noinline__ void table_add(const TableView tv, unsigned long long key, unsigned long long cnt,
@@ -114,30 +131,30 @@ static __device__ __noinline__ void table_add(const TableView tv, unsigned long 
     unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(&s->key);
     const unsigned long long f_seen = *reinterpret_cast<volatile unsigned long long*>(&s->first);
     if (k == FPX_KEY_EMPTY) {
-      k = atomicCAS(&s->key, FPX_KEY_EMPTY, key);
+      k = t_cas(tv, &s->key, FPX_KEY_EMPTY, key);
       if (k == FPX_KEY_EMPTY) {
         // this thread inserted the key: log it once (the "new combination")
-        unsigned long long pos = atomicAdd(&tv.ctl->newlog_tail, 1ull);
+        unsigned long long pos = t_add(tv, &tv.ctl->newlog_tail, 1ull);
         if (pos < tv.newlog_cap) {
           tv.newlog[pos] = key;
           tv.newlog_slot[pos] = (unsigned int)i;
         } else {
-          atomicAdd(&tv.ctl->newlog_overflow, 1ull);
+          t_add(tv, &tv.ctl->newlog_overflow, 1ull);
         }
         k = key;
       }
     }
     if (k == key) {
-      atomicAdd(&s->count, cnt);
+      t_add(tv, &s->count, cnt);
       // `first` only decreases: a value already <= ours makes the min a no-op
       // (a fresh insert reads the empty slot's ~0 and always updates).  Skips
       // most of the atomics on hot slots: all-NaN storm S1 +20 % (A/B).
-      if (first < f_seen) atomicMin(&s->first, first);
+      if (first < f_seen) t_min(tv, &s->first, first);
       return;
     }
     i = (i + 1) & tv.mask;
   }
-  atomicAdd(&tv.ctl->dropped_events, cnt);
+  t_add(tv, &tv.ctl->dropped_events, cnt);
 }
 
 // Table updates of one warp, batched: the warp-reduced (key, count, first)
@@ -151,8 +168,11 @@ struct PendingEvents {
   __device__ __forceinline__ void push(const TableView& tv, unsigned long long k, uint32_t c,
                                        unsigned long long f) {
     const uint32_t lane = threadIdx.x & 31;
-    if (n != 0 && k == last) {  // same key as the previous event: merge (first is already the smaller)
-      if (lane == n - 1) count += c;
+    if (n != 0 && k == last) {  // same key as the previous event: merge
+      if (lane == n - 1) {
+        count += c;
+        first = min(first, f);  // record paths push in index order; tensor lists need not
+      }
       return;
     }
     if (lane == n) {

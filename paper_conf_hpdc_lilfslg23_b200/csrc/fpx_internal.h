@@ -32,6 +32,11 @@ struct alignas(64) Ctl {
   unsigned long long pad[4];
 };
 
+// TableView::flags bit: the table is shared with other GPUs / processes
+// (fpx_table_export on the home handle, fpx_open_attached on the others), so
+// its atomics run at system scope (fpx_device.cuh t_cas / t_add / t_min).
+constexpr uint32_t TV_SHARED = 1u << 16;
+
 // Everything a scan kernel needs to update the table, passed by value.
 struct TableView {
   Slot* slots;
@@ -40,7 +45,7 @@ struct TableView {
   unsigned int* newlog_slot;     // slot index of each logged key (for the touched-slot reset)
   unsigned long long newlog_cap;
   Ctl* ctl;
-  uint32_t flags;                // FPX_OPT_NO_WARP_AGG (ablation) or 0
+  uint32_t flags;                // FPX_OPT_NO_WARP_AGG (ablation) | TV_SHARED
 };
 
 // One tensor of a fused multi-tensor scan (host-prepared, device-resident).

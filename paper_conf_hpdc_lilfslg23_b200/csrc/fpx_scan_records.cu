@@ -31,6 +31,7 @@
 
 #include <algorithm>
 #include <cstdlib>
+#include <mutex>
 
 #include "fpx_records.cuh"
 
@@ -470,7 +471,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     uint32_t force_any = 0u;
     if (__any_sync(FULL, in_tile && (!ok || force))) {
       const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
-      if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
+      if (bad != 0u && lane == 0) t_add(tv, &tv.ctl->bad_records, (unsigned long long)__popc(bad));
       force_any = __ballot_sync(FULL, in_tile && force);
     }
     const uint32_t my_planes = ni << (fmt == FPX_FP64 ? 1u : 0u);  // = planes_of_items(c8)
@@ -620,19 +621,30 @@ static_assert(sizeof(WarpSmem<Ring2>) % 128 == 0 && ring_smem<Ring0>() <= 227 * 
                   ring_smem<Ring2>() <= 227 * 1024 && ring_smem<Ring3>() <= 227 * 1024,
               "ring exceeds shared memory");
 
+constexpr int kMaxDevices = 64;
+
 template <int MODE, class C>
 cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uint64_t arena_planes, uint64_t base_index,
                         const TableView& tv, int num_sms, unsigned int* sched_ctr, const SchedCfg& scfg,
                         cudaStream_t s) {
-  static bool attr_set[64] = {};  // per device
+  // the shared-memory opt-in, once per device and kernel instantiation;
+  // handles may live on different host threads
+  static std::once_flag once[kMaxDevices];
+  static cudaError_t once_err[kMaxDevices];
   int dev = 0;
-  cudaGetDevice(&dev);
-  if (dev >= 64 || !attr_set[dev]) {
-    cudaError_t e = cudaFuncSetAttribute(k_scan_records_tma<MODE, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)ring_smem<C>());
-    if (e != cudaSuccess) return e;
-    if (dev < 64) attr_set[dev] = true;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  auto set_attr = [] {
+    return cudaFuncSetAttribute(k_scan_records_tma<MODE, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)ring_smem<C>());
+  };
+  if (dev < kMaxDevices) {
+    std::call_once(once[dev], [&] { once_err[dev] = set_attr(); });
+    e = once_err[dev];
+  } else {
+    e = set_attr();
   }
+  if (e != cudaSuccess) return e;
   // one CTA per SM; each warp a contiguous range of records (whole tiles of 32
   // where possible, so that ranges stay 512-B aligned in the header array)
   const uint64_t warps = (uint64_t)num_sms * C::WARPS;
@@ -697,7 +709,7 @@ k_scan_records_ldg(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     }
     const bool ok = inrange && record_valid<MODE>(h, arena_planes);
     const uint32_t bad = __ballot_sync(FULL, inrange && !ok);
-    if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
+    if (bad != 0u && lane == 0) t_add(tv, &tv.ctl->bad_records, (unsigned long long)__popc(bad));
     const uint32_t mask = ok ? h.y : 0u;
     bool force;
     const uint32_t cnt = item_counts<MODE>(h.z, ok && mask != 0u, force);
@@ -802,6 +814,38 @@ k_scan_records_ldg(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 }
 
 
+// Launch-shape knobs.  The product build uses the A/B-chosen constants; a
+// tuning build (-DFPX_TUNING, tools/ab_env.sh / ab_sched.sh only) reads them
+// once from the environment: FPX_RING (ring geometry), FPX_SCHED (0 static
+// ranges only, 2 no one-tile chunks), FPX_STATIC_PCT, FPX_DYN_CHUNK,
+// FPX_TAIL_TILES.
+struct Tuning {
+  int ring = -1;  // -1: by trace size
+  int sched = 1;
+  int static_pct = kStaticPct;
+  uint32_t dyn_chunk = kDynChunk, tail_tiles = kTailTiles;
+};
+#ifdef FPX_TUNING
+Tuning read_tuning() {
+  Tuning t;
+  if (const char* e = getenv("FPX_RING")) t.ring = atoi(e);
+  if (const char* e = getenv("FPX_SCHED")) t.sched = atoi(e);
+  if (const char* e = getenv("FPX_STATIC_PCT")) t.static_pct = std::max(0, std::min(100, atoi(e)));
+  if (const char* e = getenv("FPX_DYN_CHUNK")) t.dyn_chunk = (uint32_t)(std::max(1, atoi(e) / TILE) * TILE);
+  if (const char* e = getenv("FPX_TAIL_TILES")) t.tail_tiles = (uint32_t)std::max(0, atoi(e));
+  return t;
+}
+const Tuning& tuning() {
+  static const Tuning t = read_tuning();  // thread-safe initialisation (C++11 magic static)
+  return t;
+}
+#else
+const Tuning& tuning() {
+  static const Tuning t;
+  return t;
+}
+#endif
+
 template <int MODE>
 cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena, uint64_t arena_planes,
                              uint64_t base_index, const TableView& tv, int num_sms, uint32_t variant,
@@ -817,42 +861,18 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   }
   // Ring geometry, from interleaved A/B runs on B200 (tools/ab_env.sh,
   // profiles/r1/ab_rings.txt): 20 warps x 2 stages x 40 planes by default;
-  // 12-warp rings with 64-plane or 3-deep stages lose 10-15 %.  FPX_RING
-  // (environment, tuning only) overrides.
-  static int forced = -2;
-  if (forced == -2) {
-    const char* e = getenv("FPX_RING");
-    forced = e ? atoi(e) : -1;
-  }
-  int ring = forced;
+  // 12-warp rings with 64-plane or 3-deep stages lose 10-15 %.
   // The 24-warp ring for small traces, which are latency-bound: every warp
   // gets at most one tile up to 24 x 32 records per SM (C1: 30 us instead of
   // 45 us).  On large one-plane traces the 20-warp ring wins C5 by 2.8 % (the
   // 24-warp build is capped at 80 registers and spills) and loses the 1 %
   // NaN storm S2 by 11 % (its exact path wants more warps): the common case
   // decides.
+  const Tuning& tu = tuning();
+  int ring = tu.ring;
   if (ring < 0) ring = n <= (uint64_t)num_sms * 24 * TILE ? 3 : 1;
-  // FPX_SCHED (environment, A/B only): 0 = static ranges, 2 = no one-tile
-  // chunks at the end; default 1
-  static int sched_env = -2;
-  if (sched_env == -2) {
-    const char* e = getenv("FPX_SCHED");
-    sched_env = e ? atoi(e) : 1;
-  }
-  if (sched_env == 0) sched_ctr = nullptr;
-  // FPX_STATIC_PCT / FPX_DYN_CHUNK / FPX_TAIL_TILES (environment, A/B only):
-  // share of static ranges, records per big chunk, one-tile chunks per warp
-  static int static_pct = -1, dyn_chunk = -1, tail_tiles = -1;
-  if (static_pct < 0) {
-    const char* e = getenv("FPX_STATIC_PCT");
-    static_pct = e ? std::max(0, std::min(100, atoi(e))) : kStaticPct;
-    e = getenv("FPX_DYN_CHUNK");
-    dyn_chunk = e ? std::max(1, atoi(e) / TILE) * TILE : (int)kDynChunk;
-    e = getenv("FPX_TAIL_TILES");
-    tail_tiles = e ? std::max(0, atoi(e)) : (int)kTailTiles;
-  }
-  if (sched_env == 2) tail_tiles = 0;
-  const SchedCfg scfg{static_pct, (uint32_t)dyn_chunk, (uint32_t)tail_tiles};
+  if (tu.sched == 0) sched_ctr = nullptr;
+  const SchedCfg scfg{tu.static_pct, tu.dyn_chunk, tu.sched == 2 ? 0u : tu.tail_tiles};
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   switch (ring) {
     case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, s);

@@ -198,14 +198,11 @@ class Handle:
     def fetch(self, flags: int = FETCH_ALL, capacity: int | None = None) -> np.ndarray:
         """Entries ascending by key.  Sticky device statuses (bad record, table
         full) are kept in self.last_status, not raised."""
-        n = ctypes.c_uint64(0)
-        st = check(lib.fpx_table_fetch(self._h, None, 0, ctypes.byref(n), flags), "fpx_table_fetch",
-                   allow=(ERR_TRUNCATED, ERR_BAD_RECORD, ERR_TABLE_FULL))
-        if flags == FETCH_NEW:
-            # the first call consumed the cursor: it counted but wrote nothing,
-            # so the keys are re-read below with FETCH_ALL semantics restricted
-            # to what it returned.  Use fetch_new() instead.
+        if flags != FETCH_ALL:
             raise ValueError("use Handle.fetch_new() for FPX_FETCH_NEW")
+        n = ctypes.c_uint64(0)
+        check(lib.fpx_table_fetch(self._h, None, 0, ctypes.byref(n), flags), "fpx_table_fetch",
+              allow=(ERR_TRUNCATED, ERR_BAD_RECORD, ERR_TABLE_FULL))
         cap = n.value if capacity is None else capacity
         out = np.zeros(max(cap, 1), dtype=ENTRY_DTYPE)
         st = check(lib.fpx_table_fetch(self._h, out.ctypes.data, cap, ctypes.byref(n), flags), "fpx_table_fetch",
@@ -214,7 +211,9 @@ class Handle:
         return out[: min(cap, n.value)]
 
     def fetch_new(self, capacity: int = 1 << 20) -> np.ndarray:
-        """Keys first inserted since the previous fetch_new (FPX_FETCH_NEW)."""
+        """Keys first inserted since the previous fetch_new (FPX_FETCH_NEW), at
+        most `capacity` of them in insertion order (sorted by key); a truncated
+        call leaves the rest for the next one (last_status = ERR_TRUNCATED)."""
         n = ctypes.c_uint64(0)
         out = np.zeros(max(capacity, 1), dtype=ENTRY_DTYPE)
         st = check(lib.fpx_table_fetch(self._h, out.ctypes.data, capacity, ctypes.byref(n), FETCH_NEW),

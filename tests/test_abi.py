@@ -177,3 +177,14 @@ def test_header_is_plain_c_and_links(tmp_path):
     assert out.returncode == 0, out.stderr
     a, b = out.stdout.strip().split("|")
     assert a and b and a != b
+
+
+def test_shared_tables_use_system_scope_atomics():
+    """A table shared across GPUs (fpx_table_export / fpx_open_attached) is
+    updated from several devices at once: the library carries system-scope
+    CAS / ADD / MIN for it next to the device-scope ones of local tables
+    (CUDA memory model: an atomic is atomic only within its scope)."""
+    sass = subprocess.run(["cuobjdump", "-sass", LIB], capture_output=True, text=True, check=True).stdout
+    for op in ("CAS", "ADD", "MIN"):
+        assert re.search(rf"ATOMG?\.E\.{op}\.64\.STRONG\.SYS", sass), op
+        assert re.search(rf"ATOMG?\.E\.{op}\.64\.STRONG\.GPU", sass), op

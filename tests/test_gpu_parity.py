@@ -512,3 +512,67 @@ def test_dynamic_tail_relaunch_and_streams(fpx):
         torch.cuda.synchronize()
         got = table_dict(h.fetch())
         assert got == {k: [4 * c, f] for k, (c, f) in exp.items()}
+
+
+def test_scan_tensors_duplicate_sites_decreasing_bases_two_streams(fpx):
+    """fpx_scan_tensors == the oracle when several descriptors share (site,
+    fmt) with base indices in decreasing order (the merged event keeps the
+    smaller first index), and when back-to-back calls on two streams reuse
+    the library's descriptor buffer while the earlier launch may still run."""
+    g = torch.Generator(device=DEV).manual_seed(3)
+    items = []
+    for i in range(12):
+        t = torch.randn(50_000 + 37 * i, generator=g, device=DEV)
+        t[(7 * i) % 1000] = float("nan")
+        t[-1 - i] = float("inf")
+        items.append((t, 5 + (i % 2), 10**9 - 10**6 * i))  # two sites, bases decreasing
+    ref = oracle.Table()
+    for t, site, b in items:
+        ref.scan_tensor(t.view(torch.int32).cpu().numpy(), FP32, site=site, base_index=b)
+    with fpx.Handle(0) as h:
+        h.scan_tensors(items)
+        got = h.fetch()
+    assert_same(got, ref.entries())
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    torch.cuda.synchronize()
+    with fpx.Handle(0) as h:
+        for rep in range(20):  # alternate streams; each call rewrites the descriptor table
+            h.scan_tensors(items[rep % 3::3], stream=s1 if rep % 2 else s2)
+        torch.cuda.synchronize()
+        got = table_dict(h.fetch())
+    exp = {}
+    for rep in range(20):
+        for t, site, b in items[rep % 3::3]:
+            r = oracle.Table()
+            r.scan_tensor(t.view(torch.int32).cpu().numpy(), FP32, site=site, base_index=b)
+            for k, (c, f) in table_dict(r.entries()).items():
+                e = exp.setdefault(k, [0, 2**64 - 1])
+                e[0] += c
+                e[1] = min(e[1], f)
+    assert got == exp
+
+
+def test_fetch_new_truncated_windows_lose_nothing(fpx):
+    tr = Trace()
+    for s in range(100):
+        tr.add(s, OP_FADD, FP32, 0x1, [0x7FC00000], [])
+    hdr, arena = tr.arrays()
+    d_hdr, d_arena = to_dev(hdr, arena)
+    with fpx.Handle(0) as h:
+        h.scan_records(d_hdr, d_arena)
+        seen = []
+        while True:
+            part = h.fetch_new(capacity=30)
+            if len(part) == 0:
+                break
+            assert h.last_status in (fpx.OK, fpx.ERR_TRUNCATED)
+            seen += [int(e["site"]) for e in part]
+        assert sorted(seen) == list(range(100))  # each new key exactly once
+        with pytest.raises(ValueError):
+            h.fetch(flags=fpx.FETCH_NEW)
+        tr2 = Trace()
+        tr2.add(500, OP_FADD, FP32, 0x1, [0x7F800000], [])
+        h2, a2 = tr2.arrays()
+        d2, da2 = to_dev(h2, a2)
+        h.scan_records(d2, da2)
+        assert [int(e["site"]) for e in h.fetch_new(capacity=30)] == [500]

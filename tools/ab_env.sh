@@ -4,6 +4,7 @@
 set -u
 OUT=gpurun_out/${TAG:-abenv}; mkdir -p $OUT
 python __graft_entry__.py build > /dev/null 2>&1
+bash tools/build_tuning.sh && export FPX_LIB=$PWD/build/libfpx_tuning.so
 IFS=';' read -ra V <<< "$ENVS"
 for r in $(seq 1 ${ROUNDS:-3}); do
   for i in "${!V[@]}"; do

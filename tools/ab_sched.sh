@@ -6,6 +6,7 @@
 set -u
 O=gpurun_out/${TAG:-dyn}; mkdir -p $O
 python __graft_entry__.py build > $O/build.log 2>&1 || { tail -20 $O/build.log; exit 1; }
+bash tools/build_tuning.sh && export FPX_LIB=$PWD/build/libfpx_tuning.so
 if [ "${TESTS:-1}" = 1 ]; then
   timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_fullsize.py tests/test_gpu_fullsize_configs.py -x -q --timeout 600 > $O/pytest.log 2>&1; echo "pytest rc=$?"; tail -5 $O/pytest.log
 fi
