@@ -55,6 +55,11 @@ CONFIGS = {
                recipe=4, n=10_000_000, sites=200, p_fp64=0.0, mode=0, n_inj=0, dense=0.01),
     "c5": dict(name="C5 shard: FP32 dest-only trace, 10^11 lane-values / 8 GPUs = 3.9e8 records per GPU, 1e6 sites",
                recipe=1, n=390_625_000, sites=1_000_000, p_fp64=0.0, mode=0, rho=1e-6),
+    # at P = 1 the full C5 trace (450 GB) is scanned as
+    # regenerated chunks, scan time only -- T1 of the scaling efficiency T1/(P T_P)
+    "c5full": dict(name="C5 at P=1: the whole FP32 dest-only trace, 10^11 lane-values = 3.125e9 records over 1e6 "
+                        "sites, scanned as 8 regenerated in-HBM chunks of 3.9e8 records (scan time only)",
+                   recipe=1, n=3_125_000_000, sites=1_000_000, p_fp64=0.0, mode=0, rho=1e-6, chunks=8),
 }
 
 
@@ -69,7 +74,10 @@ PAPER_CONTEXT = {
 
 
 def config_seed(name: str) -> int:
-    """The seed of a config's synthetic input (0x5EED0000 + config)."""
+    """The seed of a config's synthetic input (0x5EED0000 + config).
+    c5full is the same trace as the c5 shards (rank r's shard = chunk r)."""
+    if name == "c5full":
+        name = "c5"
     return 0x5EED0000 + list(CONFIGS).index(name) + 1
 
 
@@ -208,9 +216,42 @@ def build_trace(cfg, rank, world, seed):
     return p, hdr, arena, planes, r0, inj
 
 
+def cpu_model() -> str:
+    """The host CPU's model name (lscpu's "Model name", from /proc/cpuinfo)."""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+class PinnedToOneCore:
+    """SURVEY §8(d) oracle-1c: the single-thread oracle pinned to one core
+    with sched_setaffinity for the duration of the timing."""
+
+    def __enter__(self):
+        self.prev = os.sched_getaffinity(0)
+        self.core = min(self.prev)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *a):
+        os.sched_setaffinity(0, self.prev)
+
+
 def cpu_baseline_oracle(cfg, seed, budget_s: float = 12.0):
     """The oracle (never tuned) on a bounded prefix of the same trace, single
-    thread on this box's host cores: lane-values/s."""
+    thread pinned to one host core of this box: lane-values/s."""
     import fpxgen
     import oracle
 
@@ -220,17 +261,20 @@ def cpu_baseline_oracle(cfg, seed, budget_s: float = 12.0):
         _, w = fpxgen.plan_injections(p, max(1, int(round(cfg.get("rho", 1e-6) * n * 32))), flow=cfg["mode"] == 1)
         fpxgen.apply_host(w, hdr, arena)
         t = oracle.Table()
-        t0 = time.perf_counter()
-        t.scan_records(hdr, arena, base_index=0, mode=cfg["mode"])
-        dt = time.perf_counter() - t0
-        return t.lane_values, dt, (hdr.nbytes + arena.nbytes) / n
+        with PinnedToOneCore() as pin:
+            t0 = time.perf_counter()
+            t.scan_records(hdr, arena, base_index=0, mode=cfg["mode"])
+            dt = time.perf_counter() - t0
+        return t.lane_values, dt, (hdr.nbytes + arena.nbytes) / n, pin.core
 
-    lv, dt, _ = run(20_000)
+    lv, dt, _, _ = run(20_000)
     n = int(min(cfg["n"], max(20_000, 20_000 * budget_s / max(dt, 1e-6))))
-    lv, dt, bpr = run(n)
+    lv, dt, bpr, core = run(n)
     return {"value": lv / dt, "unit": UNIT, "cores": 1, "kind": "oracle", "bytes_per_record": bpr,
+            "cpu_model": cpu_model(), "pinned_core": core,
             "sample": f"first {n} records of the same {cfg['name'].split(':')[0]} trace (same seed), "
-                      f"single-threaded C++ oracle, {dt:.1f} s, {lv} lane-values"}
+                      f"single-threaded C++ oracle pinned to core {core} (sched_setaffinity), scan only, "
+                      f"{dt:.1f} s, {lv} lane-values"}
 
 
 def cpu_baseline_oracle_nc(cfg, seed, single, mem_budget=12e9):
@@ -263,11 +307,12 @@ def cpu_baseline_oracle_nc(cfg, seed, single, mem_budget=12e9):
     dt_merge = time.perf_counter() - t0
     lv = sum(r[0] for r in res)
     dt = max(r[1] for r in res) + dt_merge
-    return {"value": lv / dt, "unit": UNIT, "cores": procs, "kind": "oracle",
+    return {"value": lv / dt, "unit": UNIT, "cores": procs, "kind": "oracle", "cpu_model": cpu_model(),
             "sample": f"{procs} processes x {per} records (contiguous shards of the same "
                       f"{cfg['name'].split(':')[0]} trace, same seed), unmodified C++ oracle per process, slowest "
                       f"shard {max(r[1] for r in res):.2f} s + host merge {dt_merge:.3f} s, {lv} lane-values",
-            "single_core": {"value": single["value"], "cores": 1, "sample": single["sample"]}}
+            "single_core": {"value": single["value"], "cores": 1, "pinned_core": single["pinned_core"],
+                            "sample": single["sample"]}}
 
 
 def run_reference(args, cfg, seed):
@@ -340,7 +385,8 @@ def run_reference(args, cfg, seed):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt_total / args.steps,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
         "config": {"workload": cfg["name"], "records_per_step": n * procs, "mode": ["dest", "flow"][cfg["mode"]]},
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": procs, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": procs, "kind": "oracle", "cpu_model": cpu_model(),
+                         "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -375,7 +421,8 @@ def run_reference_tensor(args, cfg, seed):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt_total / args.steps,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u16", "data": "synthetic",
         "config": {"workload": cfg["name"], "elements_per_step": n},
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "cpu_model": cpu_model(),
+                         "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
     return 0
@@ -416,6 +463,82 @@ class RecordsWorkload:
     def config(self):
         return {"records_per_gpu": self.cfg["n"], "sites": self.cfg["sites"],
                 "mode": ["dest", "flow"][self.cfg["mode"]], "planted_events": int(len(self.inj))}
+
+    def cpu_baseline(self):
+        single = cpu_baseline_oracle(self.cfg, self.seed)
+        if (os.cpu_count() or 1) == 1:
+            single.pop("bytes_per_record")
+            return single
+        return cpu_baseline_oracle_nc(self.cfg, self.seed, single)
+
+
+class ChunkedRecordsWorkload:
+    """c5full: a trace larger than HBM (450 GB) scanned as regenerated chunks
+    (SURVEY §8(d) "at P = 1 ... scanned as regenerated chunks").  Chunk c holds
+    global records [c*m, (c+1)*m) (the c5 shard of rank c), generated in HBM
+    and planted, then scanned with base_index = c*m; only the scans are timed
+    (CUDA events around each chunk's scan), the regeneration is not."""
+
+    chunked = True
+
+    def __init__(self, cfg, rank, seed, variant):
+        self.cfg, self.seed = cfg, seed
+        self.chunks = cfg["chunks"]
+        self.m = cfg["n"] // self.chunks
+        assert self.m * self.chunks == cfg["n"]
+        self.kernel = "k_scan_records_" + variant
+        self.lane_values, self.nbytes, self.planted = 0, 0, 0
+        self.scan_ms = []  # per chunk scan, last step
+        self._buf = None
+        # workload statistics of every chunk (one generation pass)
+        for c in range(self.chunks):
+            self._make(c)
+            lv, nb = workload_stats(self._buf[0], cfg["mode"])
+            self.lane_values += lv
+            self.nbytes += nb
+            self.planted += len(self._inj)
+        self._cur = self.chunks - 1
+
+    def _make(self, c):
+        import fpxgen
+
+        cfg = self.cfg
+        p = fpxgen.Params(seed=self.seed, n_records=self.m, n_sites=cfg["sites"], recipe=cfg["recipe"],
+                          p_fp64=cfg["p_fp64"])
+        self._buf = None  # free the previous chunk first (two would not fit at once)
+        hdr, arena, planes = fpxgen.generate_device(p, r0=c * self.m)
+        inj, writes = fpxgen.plan_injections(p, int(round(cfg["rho"] * self.m * 32)), r0=c * self.m)
+        fpxgen.apply_device(writes, hdr, arena)
+        self._buf, self._inj, self._planes, self._cur = (hdr, arena), inj, planes, c
+
+    def scan(self, h, stream):
+        """One step = every chunk: regenerate (untimed), scan (timed)."""
+        import torch
+
+        self.scan_ms = []
+        order = [self._cur] + [c for c in range(self.chunks) if c != self._cur]  # reuse the resident chunk first
+        evs = []
+        for c in order:
+            if c != self._cur:
+                torch.cuda.synchronize()
+                self._make(c)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            hdr, arena = self._buf
+            h.scan_records(hdr, arena, base_index=c * self.m, mode=self.cfg["mode"], stream=stream, n_records=self.m,
+                           arena_planes=self._planes)
+            b.record(stream)
+            evs.append((a, b))
+            torch.cuda.synchronize()  # the next regeneration overwrites this chunk
+        self.scan_ms = [a.elapsed_time(b) for a, b in evs]
+
+    def config(self):
+        return {"records_total": self.cfg["n"], "chunks": self.chunks, "records_per_chunk": self.m,
+                "sites": self.cfg["sites"], "mode": "dest", "planted_events": int(self.planted),
+                "timed": "sum of the chunk scans (regeneration of each chunk in HBM is outside the timed region)"}
+
+    def make_host_copies(self):
+        raise NotImplementedError("c5full (450 GB) has no host copy: e2e is measured on c5")
 
     def cpu_baseline(self):
         single = cpu_baseline_oracle(self.cfg, self.seed)
@@ -522,7 +645,7 @@ def main():
     args.warmup = max(args.warmup, 3)
     cfg = dict(CONFIGS[args.config])
     if args.records:
-        cfg["n"] = args.records
+        cfg["n"] = args.records - args.records % cfg.get("chunks", 1)
     seed = config_seed(args.config)
 
     if args.impl == "reference":
@@ -552,8 +675,11 @@ def main():
     stream = torch.cuda.current_stream(dev)
     if cfg.get("kind") == "tensor":
         wl = TensorWorkload(cfg, rank, seed, dev)
+    elif cfg.get("chunks"):
+        wl = ChunkedRecordsWorkload(cfg, rank, seed, args.variant)
     else:
         wl = RecordsWorkload(cfg, rank, seed, args.variant)
+    chunked = getattr(wl, "chunked", False)
     torch.cuda.synchronize()
 
     shared, merge_note = None, None
@@ -597,6 +723,8 @@ def main():
     if wl.nbytes < 2 * L2_BYTES:
         flush = torch.zeros(2 * L2_BYTES // 4, dtype=torch.int32, device=dev)
         sevs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    bounds = [torch.cuda.Event(enable_timing=True) for _ in range(K + 1)]
+    chunk_ms = []  # chunked workload: per step, the scan time of every chunk
     with ClockSampler(local) as clk:
         torch.cuda.synchronize()
         if world > 1:
@@ -606,24 +734,39 @@ def main():
             if flush is not None:
                 flush.add_(1)
                 sevs[i][0].record(stream)
+            bounds[i].record(stream)
             step(*evs[i])
             if flush is not None:
                 sevs[i][1].record(stream)
+            if chunked:
+                chunk_ms.append(list(wl.scan_ms))
+        bounds[K].record(stream)
         t_end.record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    total_ms = t_start.elapsed_time(t_end) if flush is None else sum(a.elapsed_time(b) for a, b in sevs)
-    kern_ms = float(np.mean([a.elapsed_time(b) for a, b in evs]))
+    if chunked:  # scan time only: the chunks' regeneration is not part of a step
+        step_ms = [sum(c) for c in chunk_ms]
+        kern_ms = float(np.mean([x for c in chunk_ms for x in c]))
+    else:
+        step_ms = ([a.elapsed_time(b) for a, b in sevs] if flush is not None else
+                   [bounds[i].elapsed_time(bounds[i + 1]) for i in range(K)])
+        kern_ms = float(np.mean([a.elapsed_time(b) for a, b in evs]))
+    total_ms = t_start.elapsed_time(t_end) if (flush is None and not chunked) else sum(step_ms)
+    median_ms = float(np.median(step_ms))
     per_rank = None
+    lane_values, nbytes = wl.lane_values, wl.nbytes
     if world > 1:
+        # max over ranks for the times; the work is summed over ranks (each
+        # rank scans its own shard)
         tdev = torch.device("cpu") if dist.get_backend() == "gloo" else dev
-        t = torch.zeros(world, 2, dtype=torch.float64, device=tdev)
-        t[rank, 0], t[rank, 1] = total_ms, kern_ms
+        t = torch.zeros(world, 5, dtype=torch.float64, device=tdev)
+        t[rank, 0], t[rank, 1], t[rank, 2], t[rank, 3], t[rank, 4] = total_ms, kern_ms, median_ms, lane_values, nbytes
         dist.all_reduce(t, op=dist.ReduceOp.SUM)  # each rank fills its own row
         per_rank = {"step_ms": [round(float(v) / K, 4) for v in t[:, 0]],
                     "scan_kernel_ms": [round(float(v), 4) for v in t[:, 1]]}
-        total_ms, kern_ms = float(t[:, 0].max()), float(t[:, 1].max())
+        total_ms, kern_ms, median_ms = float(t[:, 0].max()), float(t[:, 1].max()), float(t[:, 2].max())
+        lane_values, nbytes = int(t[:, 3].sum()), int(t[:, 4].sum())
     ms_per_step = total_ms / K
 
     if shared is None or rank == 0:
@@ -640,7 +783,9 @@ def main():
     # merged table on rank 0 in host memory (shared table: rank 0's fetch;
     # NCCL merge: the merged arrays copied to the host); time = max over ranks.
     e2e = None
-    if not args.no_e2e:
+    if chunked:
+        e2e = {"value": None, "unit": UNIT, "note": "a 450 GB trace has no host copy to stream in; e2e is on c5"}
+    elif not args.no_e2e:
         try:
             wl.make_host_copies()
             torch.cuda.synchronize()
@@ -678,12 +823,11 @@ def main():
                 dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
                 dist.all_reduce(t, op=dist.ReduceOp.SUM)
                 tot, h2d, d2h = float(tmax[0]), int(t[1]), int(t[2])
-            e2e = {"value": world * wl.lane_values / (tot / args.e2e_steps / 1e3), "unit": UNIT,
+            e2e = {"value": lane_values / (tot / args.e2e_steps / 1e3), "unit": UNIT,
                    "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "steps": args.e2e_steps}
             wl.drop_host_copies()
         except Exception as ex:  # pragma: no cover - reported, not hidden
             e2e = {"value": None, "unit": UNIT, "error": str(ex)[:200]}
-    lane_values, nbytes = wl.lane_values, wl.nbytes
 
     if rank != 0:
         if shared is not None:
@@ -693,7 +837,10 @@ def main():
         return 0
 
     peak, peak_src = load_peak()
-    achieved = nbytes / (kern_ms / 1e3) / 1e9
+    # per GPU: one launch's algorithmic bytes (the average shard; a chunk for
+    # the chunked workload) / the launch time (max over ranks)
+    launches_per_step = getattr(wl, "chunks", 1)
+    achieved = nbytes / world / launches_per_step / (kern_ms / 1e3) / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
@@ -704,12 +851,13 @@ def main():
     cpu = None if (args.no_cpu_baseline or world > 1) else wl.cpu_baseline()  # rank 0 at N = 1 only
     line = {
         "metric": METRIC,
-        "value": world * lane_values / (ms_per_step / 1e3),
+        "value": lane_values / (ms_per_step / 1e3),
         "unit": UNIT,
         "n_gpus": world,
         "steps": K,
         "warmup": args.warmup,
         "ms_per_step": ms_per_step,
+        "ms_per_step_median": median_ms,
         "higher_is_better": True,
         "scaling": "weak",
         "vs_baseline": None,
@@ -718,8 +866,9 @@ def main():
         "config": {
             "workload": cfg["name"],
             **wl.config(),
-            "lane_values_per_gpu_step": lane_values,
-            "algorithmic_bytes_per_gpu_step": nbytes,
+            "lane_values_per_step": lane_values,
+            "algorithmic_bytes_per_step": nbytes,
+            "work_summed_over_ranks": world > 1,
             "table_entries": int(len(ents)),
             "fetch_status": int(ok_status),
             "l2": ("inputs >> 126 MB L2 (no flush needed)" if flush is None else
@@ -747,7 +896,7 @@ def main():
         # per step: table reset (2 kernels) + scan (1); merge (N > 1): compact, iota,
         # radix sort, gather, sort, select-init, select, lookup (counted with ncu,
         # tools/count_merge_launches.py); NCCL's own kernels are not ours
-        "gpu_launches": K * (3 + (8 if (world > 1 and shared is None) else 0)),
+        "gpu_launches": K * (2 + launches_per_step + (8 if (world > 1 and shared is None) else 0)),
         "cpu_baseline": cpu,
         "e2e": e2e,
         **({"per_rank": per_rank} if per_rank else {}),

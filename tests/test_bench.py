@@ -52,7 +52,9 @@ def test_product_arm_json_line():
     r = d["roofline"]
     assert r["bound"] == "hbm" and r["unit"] == "GB/s" and abs(r["frac"] - r["achieved"] / r["peak"]) < 1e-9
     assert d["gpu_launches"] == 5 * 3
+    assert d["ms_per_step_median"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+    assert d["cpu_baseline"]["cpu_model"] and "pinned_core" in d["cpu_baseline"].get("single_core", d["cpu_baseline"])
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert {"sm_mhz", "sm_max_mhz", "reasons"} <= set(d["clocks"])
     assert d["config"]["fetch_status"] == 0 and d["config"]["table_entries"] > 0
@@ -75,4 +77,18 @@ def test_two_ranks_on_one_gpu(merge):
     assert d["cpu_baseline"] is None
     # e2e at N = 2: both shards copied from host memory, merged table read back on rank 0
     assert d["e2e"]["value"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
-    assert d["e2e"]["h2d_bytes_per_step"] >= 2 * d["config"]["algorithmic_bytes_per_gpu_step"]
+    assert d["config"]["work_summed_over_ranks"] is True
+    assert d["e2e"]["h2d_bytes_per_step"] >= d["config"]["algorithmic_bytes_per_step"]
+
+
+@pytest.mark.gpu
+def test_chunked_full_trace_json_line():
+    """c5full (the whole C5 trace at P = 1, regenerated chunk by chunk; scan
+    time only) at a reduced size: 8 chunks, one scan launch per chunk."""
+    lines = run(["bench.py", "--config", "c5full", "--records", "8000000", "--steps", "3", "--warmup", "3",
+                 "--no-cpu-baseline"])
+    d = lines[0]
+    assert d["config"]["chunks"] == 8 and d["config"]["records_per_chunk"] == 1_000_000
+    assert d["gpu_launches"] == 3 * (2 + 8)
+    assert d["e2e"]["value"] is None and d["value"] > 0
+    assert d["config"]["table_entries"] > 0 and d["config"]["fetch_status"] == 0
