@@ -186,13 +186,14 @@ typedef struct {
   uint32_t flags;             /* 0, or FPX_OPT_* below (ablations) */
 } fpx_options;
 
-/* Option flags, both ablations that compute the same table:
+/* Option flags.  FPX_OPT_LIVE_NEW enables early notification (fpx_poll_new
+ * below).  The other two are ablations that compute the same table:
  * FPX_OPT_SCAN_LDG selects the register-staged LDG record-scan kernel instead
  * of the default TMA (cp.async.bulk) shared-memory ring.
  * FPX_OPT_NO_WARP_AGG turns off warp aggregation (Alg2) in the
  * record scans' exact path: every lane issues its own table updates, one per
  * distinct code it holds (SURVEY §8(d) stress ablation; record scans only). */
-enum { FPX_OPT_SCAN_LDG = 1, FPX_OPT_NO_WARP_AGG = 2 };
+enum { FPX_OPT_SCAN_LDG = 1, FPX_OPT_NO_WARP_AGG = 2, FPX_OPT_LIVE_NEW = 4 };
 
 typedef struct {
   uint64_t bad_records;       /* records skipped by validation (sticky, cumulative) */
@@ -300,6 +301,25 @@ fpx_status fpx_table_merge_device(fpx_handle h, const uint64_t* d_keys, const ui
 /* Clear the table, the new-key log, its cursor and the sticky counters
  * (async on `stream`). */
 fpx_status fpx_table_reset(fpx_handle h, void* stream);
+
+/* Early notification, without waiting for scans (§3.1.2: new
+ * exceptions are pushed to the host so that users are alerted "before
+ * (hour-long) GPU runs finish").  On a handle opened with FPX_OPT_LIVE_NEW,
+ * the thread whose insert creates a key also publishes it to a ring in mapped
+ * pinned host memory (one 32-B slot per new-key-log position; capacity =
+ * newlog_capacity).  fpx_poll_new copies the keys published since the previous
+ * poll, in insertion order, into host_out (at most `capacity`; *n_out = number
+ * written) and returns at once: it calls no CUDA API and synchronises no
+ * stream, so it may run while scans are in flight.  A polled entry's key
+ * (site, kind, flow, fmt, detail) is final; its count and first_index are
+ * those of the event that inserted the key (provisional: fpx_table_fetch
+ * gives the final values once the scans are done).  fpx_table_reset restarts
+ * the ring.  Keys first inserted by another process's attached handle
+ * (fpx_open_attached) are not published here (FETCH_NEW still reports them).
+ * This poll cursor is independent of FPX_FETCH_NEW's.  A handle is used from
+ * one host thread at a time, polls included.  Errors: FPX_ERR_INVALID (no
+ * FPX_OPT_LIVE_NEW, NULL arguments). */
+fpx_status fpx_poll_new(fpx_handle h, fpx_entry* host_out, uint64_t capacity, uint64_t* n_out);
 
 /* Synchronise and read the sticky counters. */
 fpx_status fpx_get_stats(fpx_handle h, fpx_stats* out);

@@ -45,6 +45,9 @@ struct fpx_ctx {
   // streams never share one
   unsigned int* d_sched = nullptr;
   uint32_t sched_seq = 0;
+  // early notification (FPX_OPT_LIVE_NEW): mapped pinned ring + poll cursor
+  LiveSlot* h_live = nullptr;
+  uint64_t live_cursor = 0;
 };
 constexpr uint32_t kSchedSlots = 64;
 
@@ -203,7 +206,7 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   *out = nullptr;
   fpx_options o{};
   if (opt) o = *opt;
-  if ((o.flags & ~(uint32_t)(FPX_OPT_SCAN_LDG | FPX_OPT_NO_WARP_AGG)) != 0) return FPX_ERR_INVALID;
+  if ((o.flags & ~(uint32_t)(FPX_OPT_SCAN_LDG | FPX_OPT_NO_WARP_AGG | FPX_OPT_LIVE_NEW)) != 0) return FPX_ERR_INVALID;
   if (o.table_log2_slots == 0) o.table_log2_slots = 20;
   if (o.table_log2_slots < 4 || o.table_log2_slots > 30) return FPX_ERR_INVALID;
   int ndev = 0;
@@ -235,6 +238,16 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   h->tv.mask = h->slots - 1;
   h->tv.newlog_cap = cap;
   h->tv.flags = o.flags & FPX_OPT_NO_WARP_AGG;
+  h->tv.live_gen = 1;
+  if (o.flags & FPX_OPT_LIVE_NEW) {
+    // one 32-B slot per log position in host memory the kernels write through
+    // the mapping (inserts are rare: a few PCIe writes per new key)
+    if (cudaHostAlloc(&h->h_live, sizeof(LiveSlot) * cap, cudaHostAllocMapped) != cudaSuccess)
+      return fail(FPX_ERR_NOMEM);
+    std::memset(h->h_live, 0, sizeof(LiveSlot) * cap);
+    e = cudaHostGetDevicePointer(&h->tv.live, h->h_live, 0);
+    if (e != cudaSuccess) return fail(cuda_err(e, "cudaHostGetDevicePointer"));
+  }
   e = launch_table_reset(h->tv, h->slots, nullptr);
   if (e != cudaSuccess) return fail(cuda_err(e, "launch_table_reset"));
   if (!alloc_sched(h)) return fail(FPX_ERR_NOMEM);
@@ -490,7 +503,40 @@ fpx_status fpx_table_reset(fpx_handle h, void* stream) {
   if (h->last_stream != s) CK(cudaStreamSynchronize(h->last_stream));
   CK(launch_table_reset_touched(h->tv, h->slots, s));
   h->newlog_cursor = 0;
+  // scans launched from now on publish under a new generation; ring slots of
+  // the previous table (even ones written later by scans still in flight on
+  // other streams) never match the poll's expected seq again
+  h->tv.live_gen += 1;
+  h->live_cursor = 0;
   h->last_stream = s;
+  return FPX_OK;
+}
+
+fpx_status fpx_poll_new(fpx_handle h, fpx_entry* host_out, uint64_t capacity, uint64_t* n_out) {
+  if (!h || !n_out || (capacity && !host_out)) return FPX_ERR_INVALID;
+  *n_out = 0;
+  if (!h->h_live) return FPX_ERR_INVALID;  // the handle was opened without FPX_OPT_LIVE_NEW
+  // plain loads of mapped host memory: no CUDA call, no stream synchronised
+  const unsigned long long gen = (unsigned long long)h->tv.live_gen << 32;
+  uint64_t n = 0;
+  while (n < capacity && h->live_cursor < h->tv.newlog_cap) {
+    const LiveSlot* l = h->h_live + h->live_cursor;
+    const unsigned long long seq = __atomic_load_n(&l->seq, __ATOMIC_ACQUIRE);
+    if (seq != (gen | (h->live_cursor + 1))) break;  // not published yet (log order)
+    const unsigned long long k = l->key;
+    fpx_entry e;
+    std::memset(&e, 0, sizeof e);
+    e.site = (uint32_t)(k >> 32);
+    e.fmt = (uint8_t)((k >> 4) & 3);
+    e.flow = (uint8_t)((k >> 2) & 3);
+    e.kind = (uint8_t)(k & 3);
+    e.detail = (uint8_t)((k >> 6) & 7);
+    e.count = l->count;
+    e.first_index = l->first;
+    host_out[n++] = e;
+    ++h->live_cursor;
+  }
+  *n_out = n;
   return FPX_OK;
 }
 
@@ -603,6 +649,7 @@ fpx_status fpx_close(fpx_handle h) {
       cudaFree(h->tv.ctl);
     }
     cudaFreeHost(h->h_ctl);
+    if (h->h_live) cudaFreeHost(h->h_live);
     if (h->h_list) cudaFreeHost(h->h_list);
     if (h->d_list) cudaFree(h->d_list);
     if (h->list_copied) cudaEventDestroy(h->list_copied);

@@ -138,6 +138,15 @@ static __device__ __noinline__ void table_add(const TableView tv, unsigned long 
         if (pos < tv.newlog_cap) {
           tv.newlog[pos] = key;
           tv.newlog_slot[pos] = (unsigned int)i;
+          if (tv.live != nullptr) {  // early notification: publish to the host right away
+            LiveSlot* l = tv.live + pos;
+            l->key = key;
+            l->first = first;
+            l->count = cnt;
+            __threadfence_system();  // the payload is visible to the host before seq
+            *reinterpret_cast<volatile unsigned long long*>(&l->seq) =
+                ((unsigned long long)tv.live_gen << 32) | (pos + 1ull);
+          }
         } else {
           t_add(tv, &tv.ctl->newlog_overflow, 1ull);
         }

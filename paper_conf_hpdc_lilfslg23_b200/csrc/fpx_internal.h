@@ -32,6 +32,20 @@ struct alignas(64) Ctl {
   unsigned long long pad[4];
 };
 
+// Early notification ring (FPX_OPT_LIVE_NEW): one slot per new-key-log
+// position, in mapped pinned HOST memory.  The thread that inserts a key
+// writes key / count / first, fences at system scope, then publishes
+// seq = gen << 32 | (position + 1); the host polls seq in log order without
+// synchronising any stream (fpx_poll_new).  gen changes at every table reset
+// so slots of an earlier table are never taken for new ones.
+struct alignas(32) LiveSlot {
+  unsigned long long key;
+  unsigned long long first;  // index of the inserting event (provisional first)
+  unsigned long long count;  // lane-values of the inserting event (provisional count)
+  unsigned long long seq;
+};
+static_assert(sizeof(LiveSlot) == 32, "live slot is 32 B");
+
 // TableView::flags bit: the table is shared with other GPUs / processes
 // (fpx_table_export on the home handle, fpx_open_attached on the others), so
 // its atomics run at system scope (fpx_device.cuh t_cas / t_add / t_min).
@@ -46,6 +60,8 @@ struct TableView {
   unsigned long long newlog_cap;
   Ctl* ctl;
   uint32_t flags;                // FPX_OPT_NO_WARP_AGG (ablation) | TV_SHARED
+  uint32_t live_gen;             // generation of the live ring (bumped at reset)
+  LiveSlot* live;                // device view of the live ring, or nullptr
 };
 
 // One tensor of a fused multi-tensor scan (host-prepared, device-resident).

@@ -30,6 +30,7 @@ DETAIL_CMP = 4
 FETCH_ALL, FETCH_NEW = 0, 1
 OPT_SCAN_LDG = 1
 OPT_NO_WARP_AGG = 2  # ablation: no warp aggregation in the record scans' exact path
+OPT_LIVE_NEW = 4  # early notification: new keys published to mapped host memory (fpx_poll_new)
 KEY_EMPTY = 0xFFFFFFFFFFFFFFFF
 
 ENTRY_DTYPE = np.dtype(
@@ -73,6 +74,7 @@ _SIGS = {
     "fpx_table_merge_device": ([_vp, _vp, _vp, _vp, _u64, _vp], _st),
     "fpx_table_reset": ([_vp, _vp], _st),
     "fpx_get_stats": ([_vp, ctypes.POINTER(Stats)], _st),
+    "fpx_poll_new": ([_vp, _vp, _u64, _P64], _st),
     "fpx_table_export": ([_vp, ctypes.POINTER(IpcTable)], _st),
     "fpx_open_attached": ([ctypes.c_int, ctypes.POINTER(IpcTable), ctypes.POINTER(_vp)], _st),
     "fpx_close": ([_vp], _st),
@@ -220,6 +222,15 @@ class Handle:
                    "fpx_table_fetch", allow=(ERR_TRUNCATED, ERR_BAD_RECORD, ERR_TABLE_FULL))
         self.last_status = st
         return out[: min(capacity, n.value)]
+
+    def poll_new(self, capacity: int = 4096) -> np.ndarray:
+        """Keys inserted since the previous poll, while scans may still be
+        running (fpx_poll_new; needs flags=OPT_LIVE_NEW).  count / first_index
+        are the inserting event's (provisional)."""
+        n = ctypes.c_uint64(0)
+        out = np.zeros(max(capacity, 1), dtype=ENTRY_DTYPE)
+        check(lib.fpx_poll_new(self._h, out.ctypes.data, capacity, ctypes.byref(n)), "fpx_poll_new")
+        return out[: n.value]
 
     def fetch_device(self, capacity: int | None = None, stream=None):
         """(keys, counts, firsts) as int64 device tensors, sorted by key."""
