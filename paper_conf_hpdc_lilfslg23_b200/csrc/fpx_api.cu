@@ -47,6 +47,8 @@ struct fpx_ctx {
   uint32_t sched_seq = 0;
   // early notification (FPX_OPT_LIVE_NEW): mapped pinned ring + poll cursor
   LiveSlot* h_live = nullptr;
+  LiveSlot* d_live = nullptr;  // device view of h_live
+  uint32_t live_gen = 1;       // bumped at every reset
   uint64_t live_cursor = 0;
 };
 constexpr uint32_t kSchedSlots = 64;
@@ -238,17 +240,17 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   h->tv.mask = h->slots - 1;
   h->tv.newlog_cap = cap;
   h->tv.flags = o.flags & FPX_OPT_NO_WARP_AGG;
-  h->tv.live_gen = 1;
   if (o.flags & FPX_OPT_LIVE_NEW) {
     // one 32-B slot per log position in host memory the kernels write through
     // the mapping (inserts are rare: a few PCIe writes per new key)
     if (cudaHostAlloc(&h->h_live, sizeof(LiveSlot) * cap, cudaHostAllocMapped) != cudaSuccess)
       return fail(FPX_ERR_NOMEM);
     std::memset(h->h_live, 0, sizeof(LiveSlot) * cap);
-    e = cudaHostGetDevicePointer(&h->tv.live, h->h_live, 0);
+    e = cudaHostGetDevicePointer(&h->d_live, h->h_live, 0);
     if (e != cudaSuccess) return fail(cuda_err(e, "cudaHostGetDevicePointer"));
+    h->tv.flags |= TV_LIVE;
   }
-  e = launch_table_reset(h->tv, h->slots, nullptr);
+  e = launch_table_reset(h->tv, h->slots, h->d_live, h->live_gen, nullptr);
   if (e != cudaSuccess) return fail(cuda_err(e, "launch_table_reset"));
   if (!alloc_sched(h)) return fail(FPX_ERR_NOMEM);
   e = cudaStreamSynchronize(nullptr);
@@ -501,12 +503,12 @@ fpx_status fpx_table_reset(fpx_handle h, void* stream) {
   if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   if (h->last_stream != s) CK(cudaStreamSynchronize(h->last_stream));
-  CK(launch_table_reset_touched(h->tv, h->slots, s));
+  // scans ordered after this reset publish under a new generation; ring slots
+  // of the previous table (even ones written later by scans still in flight
+  // on other streams) never match the poll's expected seq again
+  h->live_gen += 1;
+  CK(launch_table_reset_touched(h->tv, h->slots, h->d_live, h->live_gen, s));
   h->newlog_cursor = 0;
-  // scans launched from now on publish under a new generation; ring slots of
-  // the previous table (even ones written later by scans still in flight on
-  // other streams) never match the poll's expected seq again
-  h->tv.live_gen += 1;
   h->live_cursor = 0;
   h->last_stream = s;
   return FPX_OK;
@@ -517,7 +519,7 @@ fpx_status fpx_poll_new(fpx_handle h, fpx_entry* host_out, uint64_t capacity, ui
   *n_out = 0;
   if (!h->h_live) return FPX_ERR_INVALID;  // the handle was opened without FPX_OPT_LIVE_NEW
   // plain loads of mapped host memory: no CUDA call, no stream synchronised
-  const unsigned long long gen = (unsigned long long)h->tv.live_gen << 32;
+  const unsigned long long gen = (unsigned long long)h->live_gen << 32;
   uint64_t n = 0;
   while (n < capacity && h->live_cursor < h->tv.newlog_cap) {
     const LiveSlot* l = h->h_live + h->live_cursor;

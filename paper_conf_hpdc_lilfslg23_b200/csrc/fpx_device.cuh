@@ -138,14 +138,13 @@ static __device__ __noinline__ void table_add(const TableView tv, unsigned long 
         if (pos < tv.newlog_cap) {
           tv.newlog[pos] = key;
           tv.newlog_slot[pos] = (unsigned int)i;
-          if (tv.live != nullptr) {  // early notification: publish to the host right away
-            LiveSlot* l = tv.live + pos;
+          if (tv.flags & TV_LIVE) {  // early notification: publish to the host right away
+            LiveSlot* l = tv.ctl->live + pos;
             l->key = key;
             l->first = first;
             l->count = cnt;
             __threadfence_system();  // the payload is visible to the host before seq
-            *reinterpret_cast<volatile unsigned long long*>(&l->seq) =
-                ((unsigned long long)tv.live_gen << 32) | (pos + 1ull);
+            *reinterpret_cast<volatile unsigned long long*>(&l->seq) = (tv.ctl->live_gen << 32) | (pos + 1ull);
           }
         } else {
           t_add(tv, &tv.ctl->newlog_overflow, 1ull);
@@ -166,14 +165,137 @@ static __device__ __noinline__ void table_add(const TableView tv, unsigned long 
   t_add(tv, &tv.ctl->dropped_events, cnt);
 }
 
+// CTA-level pre-aggregation of table updates (dense exception storms): a
+// small open-addressed table in shared memory, keyed like the device table,
+// holding a 32-bit count and a 32-bit first-index offset (relative to the
+// launch's base index) per key.  The first sighting of a key in the CTA goes
+// straight to the device table (so the key is inserted -- and reported as
+// new, P:244 -- as early as before); later events of that key only touch
+// shared memory and reach the device table once, when the CTA's last warp
+// is done (cta_warp_done).  Alg2's "reduce before any atomic"
+// one level up: per CTA instead of per warp.  A key that finds no
+// slot within CT_PROBES probes goes straight to the device table.
+constexpr uint32_t CT_SLOTS = 512, CT_PROBES = 16;
+constexpr uint32_t CT_USABLE = CT_SLOTS - 1;  // slot CT_SLOTS - 1 holds the header (see from_image)
+constexpr uint32_t CT_NONE = 0xFFFFFFFFu;
+// A tile is "dense" (its events go through the CTA table) from this many
+// warp-reduced events (FLOW / pending batches) or records with an event
+// (DEST transposed path) on.
+#ifndef FPX_DENSE_EVENTS
+#define FPX_DENSE_EVENTS 4
+#endif
+constexpr uint32_t kDenseEvents = FPX_DENSE_EVENTS;
+struct CtaTable {
+  unsigned long long* keys;  // shared [CT_SLOTS] FPX_KEY_EMPTY when free, then the
+                             // counts [CT_SLOTS] (u32, lane-values not yet in the device table)
+                             // and the first offsets [CT_SLOTS] (u32, min first index - base);
+                             // nullptr: no CTA table (events go to the device table)
+  unsigned long long base;   // the launch's base index
+  __host__ __device__ static constexpr size_t bytes() { return CT_SLOTS * 16; }
+  __device__ __forceinline__ unsigned int* cnt() const { return reinterpret_cast<unsigned int*>(keys + CT_SLOTS); }
+  __device__ __forceinline__ unsigned int* first() const { return cnt() + CT_SLOTS; }
+  __device__ __forceinline__ bool on() const { return keys != nullptr; }
+  // The record-scan ring kernel keeps the table at the START of dynamic
+  // shared memory with its header in the last slot (key = base index,
+  // count = on, first = warps done), so the exact path finds it without any
+  // register held by the scan loop.
+  __device__ static CtaTable from_image(uint8_t* smem) {
+    const unsigned long long* k = reinterpret_cast<const unsigned long long*>(smem);
+    const unsigned int* c = reinterpret_cast<const unsigned int*>(k + CT_SLOTS);
+    return CtaTable{c[CT_USABLE] ? reinterpret_cast<unsigned long long*>(smem) : nullptr, k[CT_USABLE]};
+  }
+  // by the whole CTA, before a __syncthreads
+  __device__ void init(bool on_) const {
+    for (uint32_t i = threadIdx.x; i < CT_USABLE; i += blockDim.x) {
+      keys[i] = FPX_KEY_EMPTY;
+      cnt()[i] = 0u;
+      first()[i] = CT_NONE;
+    }
+    if (threadIdx.x == 0) {
+      keys[CT_USABLE] = base;
+      cnt()[CT_USABLE] = on_ ? 1u : 0u;
+      first()[CT_USABLE] = 0u;  // warps done (cta_warp_done)
+    }
+  }
+  // one event (any lane, divergent callers welcome); c < 2^16; requires on()
+  __device__ __forceinline__ void add(const TableView& tv, unsigned long long key, uint32_t c, unsigned long long f) const {
+    uint32_t i = (uint32_t)(hash_key(key) % CT_USABLE);
+    for (uint32_t probe = 0; probe < CT_PROBES; ++probe, i = i + 1u == CT_USABLE ? 0u : i + 1u) {
+      unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(keys + i);
+      if (k == FPX_KEY_EMPTY) {
+        k = atomicCAS(keys + i, FPX_KEY_EMPTY, key);
+        if (k == FPX_KEY_EMPTY) {  // first sighting in this CTA: the device table gets it now
+          table_add(tv, key, c, f);
+          return;
+        }
+      }
+      if (k == key) {
+        unsigned int* fi = first() + i;
+        unsigned int* ci = cnt() + i;
+        const uint32_t off = (uint32_t)(f - base);
+        if (off < *reinterpret_cast<volatile unsigned int*>(fi)) atomicMin(fi, off);
+        const uint32_t old = atomicAdd(ci, c);
+        if (old + c >= 0x80000000u) {  // keep the 32-bit count far from overflow: drain it
+          const uint32_t v = atomicExch(ci, 0u);
+          if (v) table_add(tv, key, v, base + *reinterpret_cast<volatile unsigned int*>(fi));
+        }
+        return;
+      }
+    }
+    table_add(tv, key, c, f);
+  }
+};
+
+// An event of the record-scan ring kernel's exact path: through the CTA
+// table when the kernel set one up (found in shared memory, so callers hold
+// no register for it) and the tile is dense (a storm: many events, keys that
+// repeat), else straight to the device table (sparse tiles: the insert
+// latency is what counts, and a key seldom repeats within a CTA).  Out of line: the
+// scan loop's register budget stays with the fast path.  Only for kernels
+// whose dynamic shared memory starts with a CtaTable image.
+static __device__ __noinline__ void emit_event(const TableView tv, unsigned long long key, uint32_t c,
+                                              unsigned long long f, bool dense) {
+  extern __shared__ __align__(128) uint8_t fpx_dyn_smem[];
+  const CtaTable ct = CtaTable::from_image(fpx_dyn_smem);
+  if (dense && ct.on()) ct.add(tv, key, c, f);
+  else table_add(tv, key, c, f);
+}
+
+// Called once by every warp of the ring kernel's CTA as it finishes
+// (warp-uniform).  The last one to arrive adds every slot's pending count
+// (with its min first index) to the device table: the other warps' shared
+// memory updates happen before their (fenced) arrival, so it sees them all.
+// The arrival counter is the header slot's first-offset word.  Out of line,
+// like emit_event, so the scan loop keeps no register for it.
+static __device__ __noinline__ void cta_warp_done(const TableView tv, uint32_t nwarps) {
+  extern __shared__ __align__(128) uint8_t fpx_dyn_smem[];
+  const CtaTable ct = CtaTable::from_image(fpx_dyn_smem);
+  if (!ct.on()) return;
+  const uint32_t lane = threadIdx.x & 31u;
+  __syncwarp();
+  __threadfence_block();
+  uint32_t last = 0u;
+  if (lane == 0u) last = atomicAdd(ct.first() + CT_USABLE, 1u) == nwarps - 1u ? 1u : 0u;
+  if (__shfl_sync(0xFFFFFFFFu, last, 0) == 0u) return;
+  __threadfence_block();
+  for (uint32_t i = lane; i < CT_USABLE; i += 32u) {
+    const unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(ct.keys + i);
+    const uint32_t c = *reinterpret_cast<volatile unsigned int*>(ct.cnt() + i);
+    if (k != FPX_KEY_EMPTY && c != 0u) table_add(tv, k, c, ct.base + *reinterpret_cast<volatile unsigned int*>(ct.first() + i));
+  }
+}
+
 // Table updates of one warp, batched: the warp-reduced (key, count, first)
 // events of a tile are parked one per lane and issued by up to 32 lanes at
 // once, so a dense tile (storms) costs ~one L2 round trip per 32 events
 // instead of one per event.  Consecutive events with the same key (a storm
 // over one site) merge before any atomic.  `n` and `last` are warp-uniform.
+// CTA = true: the issued events go through emit_event (CTA table).
+template <bool CTA = false>  // CTA: issue through emit_event (ring kernel only)
 struct PendingEvents {
   unsigned long long key = 0, first = 0, last = FPX_KEY_EMPTY;
   uint32_t count = 0, n = 0;
+  bool warm = false;  // CTA: the warp is in a storm; dense batches may use the CTA table
   __device__ __forceinline__ void push(const TableView& tv, unsigned long long k, uint32_t c,
                                        unsigned long long f) {
     const uint32_t lane = threadIdx.x & 31;
@@ -196,7 +318,11 @@ struct PendingEvents {
   // atomics was tried: +16 % on an all-NaN storm, -4 % / -11 % on the 1 %
   // storm and C1, so the plain per-lane issue stays.)
   __device__ __forceinline__ void flush(const TableView& tv) {
-    if ((threadIdx.x & 31) < n) table_add(tv, key, count, first);
+    const bool dense = warm && n >= kDenseEvents;  // warp-uniform
+    if ((threadIdx.x & 31) < n) {
+      if (CTA) emit_event(tv, key, count, first, dense);
+      else table_add(tv, key, count, first);
+    }
     n = 0;
     last = FPX_KEY_EMPTY;
     __syncwarp();
@@ -206,8 +332,8 @@ struct PendingEvents {
 // Warp aggregation of one record's events.  Every lane passes a bitmask of
 // the codes it holds (bit c = code c present) plus, per code, its count via
 // the `count_of` functor.  Must be called by the full warp (uniform).
-template <typename CountOf>
-__device__ __forceinline__ void warp_flush(const TableView& tv, PendingEvents& pend, uint32_t code_mask,
+template <typename CountOf, typename Pend>
+__device__ __forceinline__ void warp_flush(const TableView& tv, Pend& pend, uint32_t code_mask,
                                            uint32_t site, uint32_t fmt, unsigned long long gidx, CountOf count_of) {
   uint32_t all = __reduce_or_sync(FULL, code_mask);
   while (all) {
@@ -220,7 +346,8 @@ __device__ __forceinline__ void warp_flush(const TableView& tv, PendingEvents& p
 
 // Warp aggregation when every lane holds at most one event code (the FLOW
 // modes): lanes with equal codes are grouped with a ballot per distinct code.
-__device__ __forceinline__ void warp_flush_single(const TableView& tv, PendingEvents& pend, int code, uint32_t site,
+template <typename Pend>
+__device__ __forceinline__ void warp_flush_single(const TableView& tv, Pend& pend, int code, uint32_t site,
                                                   uint32_t fmt, unsigned long long gidx) {
   uint32_t pending = __ballot_sync(FULL, code >= 0);
   while (pending) {
@@ -230,6 +357,15 @@ __device__ __forceinline__ void warp_flush_single(const TableView& tv, PendingEv
     pend.push(tv, make_key(site, fmt, (uint32_t)c), __popc(peers), gidx);
     pending &= ~peers;
   }
+}
+
+// Shared-memory address of a generic pointer into shared memory, and a
+// 128-bit shared load at such an address.
+__device__ __forceinline__ uint32_t sh_addr(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+__device__ __forceinline__ uint4 sh_ld4(uint32_t addr) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));
+  return v;
 }
 
 // Streaming 32-bit / 128-bit loads: read-only path, no L1 allocation.

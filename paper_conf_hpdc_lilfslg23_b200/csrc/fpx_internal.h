@@ -24,12 +24,15 @@ struct alignas(32) Slot {
 };
 static_assert(sizeof(Slot) == 32, "slot = one 32-B L2 sector");
 
+struct LiveSlot;
 struct alignas(64) Ctl {
   unsigned long long bad_records;
   unsigned long long dropped_events;
   unsigned long long newlog_tail;      // number of inserts ever (= table entries)
   unsigned long long newlog_overflow;
-  unsigned long long pad[4];
+  LiveSlot* live;                      // device view of the live ring (TV_LIVE handles only)
+  unsigned long long live_gen;         // its generation, set by every reset
+  unsigned long long pad[2];
 };
 
 // Early notification ring (FPX_OPT_LIVE_NEW): one slot per new-key-log
@@ -50,6 +53,10 @@ static_assert(sizeof(LiveSlot) == 32, "live slot is 32 B");
 // (fpx_table_export on the home handle, fpx_open_attached on the others), so
 // its atomics run at system scope (fpx_device.cuh t_cas / t_add / t_min).
 constexpr uint32_t TV_SHARED = 1u << 16;
+// TableView::flags bit: this handle publishes new keys to its live ring
+// (ctl->live; FPX_OPT_LIVE_NEW on the home handle; never on attached ones,
+// whose process cannot see the home's host ring).
+constexpr uint32_t TV_LIVE = 1u << 17;
 
 // Everything a scan kernel needs to update the table, passed by value.
 struct TableView {
@@ -59,9 +66,7 @@ struct TableView {
   unsigned int* newlog_slot;     // slot index of each logged key (for the touched-slot reset)
   unsigned long long newlog_cap;
   Ctl* ctl;
-  uint32_t flags;                // FPX_OPT_NO_WARP_AGG (ablation) | TV_SHARED
-  uint32_t live_gen;             // generation of the live ring (bumped at reset)
-  LiveSlot* live;                // device view of the live ring, or nullptr
+  uint32_t flags;                // FPX_OPT_NO_WARP_AGG (ablation) | TV_SHARED | TV_LIVE
 };
 
 // One tensor of a fused multi-tensor scan (host-prepared, device-resident).
@@ -88,11 +93,13 @@ cudaError_t launch_scan_tensor(const void* d_ptr, uint64_t n_elems, uint32_t fmt
                                uint64_t base_index, const TableView& tv, int num_sms, cudaStream_t s);
 cudaError_t launch_scan_tensor_list(const ListEntry* d_entries, uint32_t n, uint64_t total_vec,
                                     uint64_t total_scalar, const TableView& tv, int num_sms, cudaStream_t s);
-cudaError_t launch_table_reset(const TableView& tv, uint64_t slots, cudaStream_t s);
+// Both resets also (re)write ctl->live / live_gen (the early-notification ring).
+cudaError_t launch_table_reset(const TableView& tv, uint64_t slots, LiveSlot* live, uint32_t live_gen, cudaStream_t s);
 // Clear only the slots recorded in the new-key log (every occupied slot is
 // there unless the log overflowed, in which case the whole table is cleared),
 // then the counters.  O(entries) instead of O(slots); stream-ordered, no sync.
-cudaError_t launch_table_reset_touched(const TableView& tv, uint64_t slots, cudaStream_t s);
+cudaError_t launch_table_reset_touched(const TableView& tv, uint64_t slots, LiveSlot* live, uint32_t live_gen,
+                                      cudaStream_t s);
 // Compact non-empty slots into (keys, counts, firsts); *d_n receives the count.
 cudaError_t launch_table_compact(const TableView& tv, uint64_t slots, uint64_t* d_keys,
                                  uint64_t* d_counts, uint64_t* d_first, unsigned long long* d_n,

@@ -161,9 +161,9 @@ __device__ __forceinline__ uint32_t eval_record(const RecDesc& d, const uint32_t
 }
 
 // Exact evaluation + warp aggregation + table update of one record.
-template <int MODE>
+template <int MODE, typename Pend>
 __device__ __forceinline__ void flush_record(const RecDesc& d, const uint32_t* __restrict__ lane_base, int lane,
-                                             uint64_t gidx, const TableView& tv, PendingEvents& pend,
+                                             uint64_t gidx, const TableView& tv, Pend& pend,
                                              const uint32_t* staged = nullptr) {
   uint32_t codes, evm;
   const uint32_t cm = eval_record<MODE>(d, lane_base, lane, codes, evm, staged);
@@ -198,7 +198,7 @@ __device__ __forceinline__ void flush_record(const RecDesc& d, const uint32_t* _
 template <int MODE>
 __device__ __noinline__ void exact_tile(const RecDesc* __restrict__ recs, const uint32_t* __restrict__ lane_base,
                                         int lane, uint64_t gidx0, const TableView tv) {
-  PendingEvents pend;
+  PendingEvents<> pend;
   for (int j = 0; j < TILE; ++j) {
     const RecDesc d = recs[j];
     if (d.mask == 0u) continue;  // warp-uniform
@@ -218,7 +218,7 @@ __device__ __noinline__ void exact_tile(const RecDesc* __restrict__ recs, const 
 template <int MODE, typename Needed>
 __device__ __forceinline__ void exact_tile_records(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
                                             const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
-                                            int lane, uint64_t gidx0, const TableView tv, Needed needed) {
+                                            int lane, uint64_t gidx0, const TableView tv, bool warm, Needed needed) {
   uint4 h = make_uint4(0u, 0u, 0u, 0u);
   if ((uint32_t)lane < k) h = hdr_tile[lane];
   const bool ok = (uint32_t)lane < k && record_valid<MODE>(h, arena_planes);
@@ -232,7 +232,8 @@ __device__ __forceinline__ void exact_tile_records(const uint4* __restrict__ hdr
   }
   slot -= c;
   const uint32_t staged_slot = c != 0u ? slot : 0xFFFFFFFFu;
-  PendingEvents pend;
+  PendingEvents<true> pend;
+  pend.warm = warm;
   for (uint32_t j = 0; j < k; ++j) {
     const RecDesc d{__shfl_sync(FULL, h.w, j), __shfl_sync(FULL, mask, j), __shfl_sync(FULL, h.z, j),
                     __shfl_sync(FULL, h.x, j)};
@@ -242,6 +243,56 @@ __device__ __forceinline__ void exact_tile_records(const uint4* __restrict__ hdr
     flush_record<MODE>(d, lane_base, lane, gidx0 + j, tv, pend, sl != 0xFFFFFFFFu ? stage_lane + sl * 32 : nullptr);
   }
   pend.flush(tv);
+}
+
+// Class counts (NaN, INF, SUB) over the active lanes' values in the `dw`
+// staged destination planes of this lane's record (plane 0 at shared
+// address sp).  Each load reads 16 B = instrumented lanes 4v..4v+3, with v
+// skewed by the lane so that each 8-lane phase of a warp's LDS.128 touches
+// all 32 banks once.  Thresholds on doubled magnitudes (the sign drops out):
+//   FP32  a = 2x:                 NaN a > 0xFF000000, INF a == 0xFF000000, SUB a - 2 < 0xFFFFFE
+//   FP64  a = 2 hi + min(lo, 1):  NaN a > 0xFFE00000, INF a == 0xFFE00000, SUB a - 1 < 0x1FFFFF
+//   FP16 / BF16 per half h = |x|: NaN h > E, INF h == E, SUB h - 1 < M (E, M = 0x7C00, 0x3FF / 0x7F80, 0x7F)
+// (the same definitions as cls_*, §2.1).
+template <uint32_t FMT>
+__device__ __forceinline__ void count_staged(uint32_t sp, uint32_t dw, uint32_t mask, uint32_t lane, uint32_t& n_nan,
+                                             uint32_t& n_inf, uint32_t& n_sub) {
+  constexpr uint32_t STEP = FMT == FPX_FP64 ? 2u : 1u;
+  for (uint32_t w = 0; w < dw; w += STEP) {
+#pragma unroll
+    for (uint32_t u = 0; u < 8; ++u) {
+      const uint32_t v = (u + lane) & 7u;
+      const uint32_t m4 = mask >> (4u * v);
+      const uint4 x = sh_ld4(sp + w * 128u + v * 16u);
+      uint32_t xs[4] = {x.x, x.y, x.z, x.w};
+      uint32_t hs[4] = {0u, 0u, 0u, 0u};
+      if (FMT == FPX_FP64) {
+        const uint4 y = sh_ld4(sp + (w + 1u) * 128u + v * 16u);
+        hs[0] = y.x, hs[1] = y.y, hs[2] = y.z, hs[3] = y.w;
+      }
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k) {
+        const bool act = (m4 >> k) & 1u;
+        if (FMT == FPX_FP32) {
+          const uint32_t a = xs[k] + xs[k];
+          n_nan += (act && a > 0xFF000000u) ? 1u : 0u;
+          n_inf += (act && a == 0xFF000000u) ? 1u : 0u;
+          n_sub += (act && a - 2u < 0x00FFFFFEu) ? 1u : 0u;
+        } else if (FMT == FPX_FP64) {
+          const uint32_t a = hs[k] * 2u + min(xs[k], 1u);
+          n_nan += (act && a > 0xFFE00000u) ? 1u : 0u;
+          n_inf += (act && a == 0xFFE00000u) ? 1u : 0u;
+          n_sub += (act && a - 1u < 0x001FFFFFu) ? 1u : 0u;
+        } else {
+          constexpr uint32_t E = FMT == FPX_FP16 ? 0x7C00u : 0x7F80u, M = FMT == FPX_FP16 ? 0x03FFu : 0x007Fu;
+          const uint32_t lo = xs[k] & 0x7FFFu, hi = (xs[k] >> 16) & 0x7FFFu;
+          n_nan += act ? (lo > E ? 1u : 0u) + (hi > E ? 1u : 0u) : 0u;
+          n_inf += act ? (lo == E ? 1u : 0u) + (hi == E ? 1u : 0u) : 0u;
+          n_sub += act ? (lo - 1u < M ? 1u : 0u) + (hi - 1u < M ? 1u : 0u) : 0u;
+        }
+      }
+    }
+  }
 }
 
 // DEST-mode exact path of a TMA tile, transposed: lane j evaluates ALL lanes of
@@ -256,7 +307,10 @@ __device__ __forceinline__ void exact_tile_records(const uint4* __restrict__ hdr
 // this lane's header, staged planes and stage slot.
 __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t mask, uint32_t c, uint32_t slot,
                                                       const uint32_t* __restrict__ arena, const uint32_t* stage,
-                                                      int lane, uint64_t gidx0, const TableView& tv) {
+                                                      int lane, uint64_t gidx0, const TableView& tv, bool warm) {
+  // group leaders' updates go through the CTA table when there is one
+  bool dense = false;  // set below, warp-uniform: warm and records of the tile with an event >= kDenseEvents
+  auto emit = [&](unsigned long long key, uint32_t cnt_, unsigned long long f) { emit_event(tv, key, cnt_, f, dense); };
   const uint32_t op = op_of(h.z), fmt = fmt_of(h.z), nsrc = nsrc_of(h.z), dw = dwords_of(h.z);
   const uint32_t sw = sw_of(fmt);
   const bool have_div = (op == FPX_OP_DIV) && nsrc >= 2 && dw == sw;
@@ -282,42 +336,29 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
       // Every other opclass maps the destination CLASS to a kind per record
       // (dest_kind: RCP -> DIV0 for NaN / INF, nothing for SUB; else the
       // class), so the loop only counts classes, per format (lanes of one
-      // format run together).  Inactive lanes are masked to 0 (clean).
+      // format run together).
       uint32_t n_nan = 0u, n_inf = 0u, n_sub = 0u;
-      switch (fmt) {
-        case FPX_FP32:
-          for (uint32_t t = 0; t < 32; ++t) {
-            const uint32_t i = (t + (uint32_t)lane) & 31u, act = 0u - ((mask >> i) & 1u);
-            for (uint32_t w = 0; w < dw; ++w) {
-              const uint32_t a = p[w * 32 + i] & act & 0x7FFFFFFFu;
-              n_nan += a > 0x7F800000u;
-              n_inf += a == 0x7F800000u;
-              n_sub += (a - 1u) < 0x007FFFFFu;
-            }
-          }
-          break;
-        case FPX_FP64:
-          for (uint32_t t = 0; t < 32; ++t) {
-            const uint32_t i = (t + (uint32_t)lane) & 31u, act = 0u - ((mask >> i) & 1u);
-            for (uint32_t w = 0; w < dw; w += 2) {
-              const uint32_t lo = p[w * 32 + i] & act, ah = p[(w + 1) * 32 + i] & act & 0x7FFFFFFFu;
-              const bool mant_nz = ((ah & 0x000FFFFFu) | lo) != 0u, exp_max = ah >= 0x7FF00000u;
-              n_nan += exp_max && mant_nz;
-              n_inf += exp_max && !mant_nz;
-              n_sub += ah < 0x00100000u && mant_nz;
-            }
-          }
-          break;
-        default: {
-          const uint32_t em = fmt == FPX_FP16 ? 0x7C00u : 0x7F80u, mm = fmt == FPX_FP16 ? 0x03FFu : 0x007Fu;
-          for (uint32_t t = 0; t < 32; ++t) {
-            const uint32_t i = (t + (uint32_t)lane) & 31u, act = 0u - ((mask >> i) & 1u);
-            for (uint32_t w = 0; w < dw; ++w) {
-              const uint32_t x = p[w * 32 + i] & act & 0x7FFF7FFFu;
-              const uint32_t lo = x & 0xFFFFu, hi = x >> 16;
-              n_nan += (lo > em) + (hi > em);
-              n_inf += (lo == em) + (hi == em);
-              n_sub += ((lo - 1u) < mm) + ((hi - 1u) < mm);
+      if (c != 0u) {
+        // staged planes: 16 B per load (count_staged)
+        const uint32_t sp = sh_addr(stage) + slot * 128u;
+        switch (fmt) {
+          case FPX_FP32: count_staged<FPX_FP32>(sp, dw, mask, (uint32_t)lane, n_nan, n_inf, n_sub); break;
+          case FPX_FP64: count_staged<FPX_FP64>(sp, dw, mask, (uint32_t)lane, n_nan, n_inf, n_sub); break;
+          case FPX_FP16: count_staged<FPX_FP16>(sp, dw, mask, (uint32_t)lane, n_nan, n_inf, n_sub); break;
+          default: count_staged<FPX_BF16>(sp, dw, mask, (uint32_t)lane, n_nan, n_inf, n_sub);
+        }
+      } else {
+        // planes in global memory (a recorded division whose destination is
+        // not one source wide, R19: not staged): the plain per-value class
+        for (uint32_t t = 0; t < 32; ++t) {
+          if (((mask >> t) & 1u) == 0u) continue;
+          for (uint32_t w = 0; w < dw; w += fmt == FPX_FP64 ? 2u : 1u) {
+            const uint32_t lo = p[w * 32 + t], hi = fmt == FPX_FP64 ? p[(w + 1) * 32 + t] : 0u;
+            for (uint32_t hv = 0; hv < (fmt >= FPX_FP16 ? 2u : 1u); ++hv) {
+              const uint32_t cl = cls_val(fmt, fmt >= FPX_FP16 ? (lo >> (16 * hv)) & 0xFFFFu : lo, hi);
+              n_nan += cl == CLS_NAN;
+              n_inf += cl == CLS_INF;
+              n_sub += cl == CLS_SUB;
             }
           }
         }
@@ -336,6 +377,7 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
   // parks its sums (one per kind it leads) and the updates of different kinds
   // and records run in parallel instead of one warp-wide round per kind (C1
   // +11 %).  A single kind (storms) updates right away (S2 -2 % otherwise).
+  dense = warm && __popc(__ballot_sync(FULL, present != 0u)) >= kDenseEvents;
   uint32_t all = __reduce_or_sync(FULL, present), lead = 0u;
   if (__popc(all) == 1) {
     const uint32_t kd = (uint32_t)(__ffs(all) - 1);
@@ -344,7 +386,7 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
     const uint32_t peers = __match_any_sync(FULL, key);
     if (has) {
       const uint32_t sum = __reduce_add_sync(peers, (uint32_t)((cnt >> (16 * kd)) & 0xFFFFu));
-      if ((uint32_t)lane == (uint32_t)(__ffs(peers) - 1)) table_add(tv, key, sum, gidx0 + (uint64_t)lane);
+      if ((uint32_t)lane == (uint32_t)(__ffs(peers) - 1)) emit(key, sum, gidx0 + (uint64_t)lane);
     }
     return;
   }
@@ -367,7 +409,7 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
   while (lead) {
     const uint32_t kd = (uint32_t)(__ffs(lead) - 1);
     lead &= lead - 1u;
-    table_add(tv, make_key(h.x, fmt, kd), (sums >> (16 * kd)) & 0xFFFFu, gidx0 + (uint64_t)lane);
+    emit(make_key(h.x, fmt, kd), (uint32_t)((sums >> (16 * kd)) & 0xFFFFu), gidx0 + (uint64_t)lane);
   }
 }
 
@@ -380,10 +422,12 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
 // storm-heavy FLOW traces: FLOW tiles hold ~10 records, so most lanes idle,
 // and per-record operand counts and formats diverge inside the loop
 // (profiles/r1/ab_sched.txt).  A/B in profiles/r1/ab_producer.txt (ab9-ab16).
+// Table updates go through emit_event (the CTA pre-aggregation table, if the
+// kernel set one up, then the device table).
 template <int MODE, typename Needed>
-__device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
+__device__ __forceinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
                                             const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
-                                            int lane, uint64_t gidx0, const TableView tv, Needed needed) {
+                                            int lane, uint64_t gidx0, const TableView tv, bool warm, Needed needed) {
   if (MODE == FPX_MODE_DEST && !(tv.flags & FPX_OPT_NO_WARP_AGG)) {
     uint4 h = make_uint4(0u, 0u, 0u, 0u);
     if ((uint32_t)lane < k) h = hdr_tile[lane];
@@ -396,10 +440,10 @@ __device__ __noinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, 
       const uint32_t t = __shfl_up_sync(FULL, slot, o);
       if (lane >= o) slot += t;
     }
-    exact_tile_transposed(h, mask, c, slot - c, lane_base - lane, stage_lane - lane, lane, gidx0, tv);
+    exact_tile_transposed(h, mask, c, slot - c, lane_base - lane, stage_lane - lane, lane, gidx0, tv, warm);
     return;
   }
-  exact_tile_records<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, needed);
+  exact_tile_records<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, warm, needed);
 }
 
 // Plane items of one record for the fast path, by list:

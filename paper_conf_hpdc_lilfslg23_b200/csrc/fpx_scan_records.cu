@@ -135,9 +135,11 @@ __device__ __forceinline__ uint32_t decode_index(uint32_t meta) { return ((meta 
 // meta bits outside the table index that a valid record keeps zero
 constexpr uint32_t META_RESERVED = 0xFFFF80E0u;
 
+// shared memory of the ring kernel: per-warp rings, the decode table, the
+// CTA pre-aggregation table (fpx_device.cuh CtaTable)
 template <class C>
 constexpr size_t ring_smem() {
-  return sizeof(WarpSmem<C>) * C::WARPS + DECODE_ENTRIES;
+  return CtaTable::bytes() + sizeof(WarpSmem<C>) * C::WARPS + DECODE_ENTRIES;
 }
 
 // Header decode for the fast path, branch-free: validity (the contract of
@@ -379,6 +381,44 @@ constexpr int kMaxWarpTimes = 148 * 32;
 __device__ unsigned long long g_warp_t0[kMaxWarpTimes], g_warp_t1[kMaxWarpTimes];
 #endif
 
+// The exact path of a hit tile (rec::exact_tile_hdr with this kernel's
+// needed-plane count).  `warm`: this warp has met enough hit tiles for the
+// CTA pre-aggregation table to pay (a storm); dense tiles then go through it.
+template <int MODE>
+__device__ __forceinline__ void exact_tile_ring(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
+                                                const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
+                                                int lane, uint64_t gidx0, const TableView tv, bool warm) {
+  exact_tile_hdr<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, warm, [](uint32_t meta) {
+    bool f;
+    const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, f, f);
+    return fmt_of(meta) == FPX_FP64 ? 2u * ni : ni;
+  });
+}
+// DEST: inlined (its transposed path fits the scan loop's registers: no
+// spill).  FLOW / FLOW_DETAIL: called through a function pointer -- a direct
+// call lets ptxas allocate caller and callee registers together and the
+// record-walking path's demands then spill the scan loop's live values (up
+// to 180 B per tile); an indirect call uses the ABI calling convention,
+// whose saves and restores sit around the call, on the rare path only.
+template <int MODE>
+__device__ __noinline__ void exact_tile_ring_call(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
+                                                  const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
+                                                  int lane, uint64_t gidx0, const TableView tv, bool warm) {
+  exact_tile_ring<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, warm);
+}
+using ExactFn = void (*)(const uint4*, uint32_t, uint64_t, const uint32_t*, const uint32_t*, int, uint64_t,
+                         const TableView, bool);
+template <int MODE>
+__device__ ExactFn g_exact_fn = exact_tile_ring_call<MODE>;
+#ifndef DESTCALL
+#define DESTCALL exact_tile_ring
+#endif
+#ifndef FLOWCALL
+#define FLOWCALL g_exact_fn
+#endif
+// the CTA table is used by a warp from its kWarmTiles-th hit tile on
+constexpr uint32_t kWarmTiles = 8;
+
 template <int MODE, class C>
 __global__ void __launch_bounds__(C::WARPS * 32, 1)
 k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __restrict__ arena,
@@ -386,15 +426,26 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
                    const TableView tv) {
   constexpr int STAGES = C::STAGES, PLANES = C::PLANES;
   static_assert(PLANES <= 64, "stage sizes keep the byte fields of the packed scan exact");
-  extern __shared__ __align__(128) uint8_t smem_raw[];
+  // dynamic shared memory: [CTA table][per-warp rings][decode table]
+  extern __shared__ __align__(128) uint8_t fpx_dyn_smem[];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  WarpSmem<C>& sm = reinterpret_cast<WarpSmem<C>*>(smem_raw)[warp];
-  uint8_t* lut = smem_raw + sizeof(WarpSmem<C>) * C::WARPS;
+  uint8_t* rings = fpx_dyn_smem + CtaTable::bytes();
+  WarpSmem<C>& sm = reinterpret_cast<WarpSmem<C>*>(rings)[warp];
+  uint8_t* lut = rings + sizeof(WarpSmem<C>) * C::WARPS;
   build_decode_table<MODE>(lut);
+  // CTA pre-aggregation of the exact path's table updates (fpx_device.cuh
+  // CtaTable; the exact path finds it through emit_event); off for the
+  // no-aggregation ablation and for launches whose record offsets need more
+  // than 32 bits
+  CtaTable{reinterpret_cast<unsigned long long*>(fpx_dyn_smem), base_index}
+      .init((tv.flags & FPX_OPT_NO_WARP_AGG) == 0u && n < (uint64_t)CT_NONE);
   __syncthreads();
   const uint64_t gw = blockIdx.x * (uint64_t)C::WARPS + warp;
   const uint64_t start = gw * recs_per_warp;
-  if (start >= n) return;  // warp-uniform; no block-wide barriers below this line
+  if (start >= n) {  // warp-uniform; no block-wide barriers below this line
+    cta_warp_done(tv, C::WARPS);
+    return;
+  }
 #ifdef FPX_WARP_TIMES
   if (lane == 0 && gw < kMaxWarpTimes) g_warp_t0[gw] = globaltimer_ns();
 #endif
@@ -412,6 +463,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 #pragma unroll
     for (int s = 0; s < STAGES; ++s) mbar_init(&sm.bar[s], 1);
     mbar_init_fence();
+    sm.meta[0].pad[0] = 0u;  // hit tiles of this warp (exact path, CTA-table warm-up)
   }
   __syncwarp();
 
@@ -471,7 +523,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     uint32_t force_any = 0u;
     if (__any_sync(FULL, in_tile && (!ok || force))) {
       const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
-      if (bad != 0u && lane == 0) t_add(tv, &tv.ctl->bad_records, (unsigned long long)__popc(bad));
+      if (bad != 0u && lane == 0) atomicAdd_system(&tv.ctl->bad_records, (unsigned long long)__popc(bad));  // rare; system scope covers shared tables
       force_any = __ballot_sync(FULL, in_tile && force);
     }
     const uint32_t my_planes = ni << (fmt == FPX_FP64 ? 1u : 0u);  // = planes_of_items(c8)
@@ -573,6 +625,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
         atomicExch(sch.ctr, 0u);
         atomicExch(sch.ctr + 1, 0u);
       }
+      cta_warp_done(tv, C::WARPS);
       break;
     }
     mbar_wait(&sm.bar[s], (phase >> s) & 1u);
@@ -602,12 +655,20 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       consume_list<FPX_BF16, true>(w, seg[7], seg[8], ia, pa, g, q);
     }
     if (__any_sync(FULL, w.hit_wide() || (halves && w.hit_half())) || (mk & kForceBit) != 0u)
-      exact_tile_hdr<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane, lane,
-                           m.gidx0, tv, [](uint32_t meta) {
-                             bool f;
-                             const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, f, f);
-                             return fmt_of(meta) == FPX_FP64 ? 2u * ni : ni;
-                           });
+    {
+      // hit tiles of this warp so far: kept in shared memory (the stage-0
+      // descriptor's spare word), not in a register of the scan loop
+      const uint32_t hits = sm.meta[0].pad[0];
+      __syncwarp();
+      if (lane == 0) sm.meta[0].pad[0] = hits + 1u;
+      const bool warm = hits >= kWarmTiles;
+      if (MODE == FPX_MODE_DEST)
+        DESTCALL<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base,
+                              sm.planes[s] + lane, lane, m.gidx0, tv, warm);
+      else
+        FLOWCALL<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
+                         lane, m.gidx0, tv, warm);
+    }
   }
 }
 
@@ -709,7 +770,7 @@ k_scan_records_ldg(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     }
     const bool ok = inrange && record_valid<MODE>(h, arena_planes);
     const uint32_t bad = __ballot_sync(FULL, inrange && !ok);
-    if (bad != 0u && lane == 0) t_add(tv, &tv.ctl->bad_records, (unsigned long long)__popc(bad));
+    if (bad != 0u && lane == 0) atomicAdd_system(&tv.ctl->bad_records, (unsigned long long)__popc(bad));  // rare; system scope covers shared tables
     const uint32_t mask = ok ? h.y : 0u;
     bool force;
     const uint32_t cnt = item_counts<MODE>(h.z, ok && mask != 0u, force);

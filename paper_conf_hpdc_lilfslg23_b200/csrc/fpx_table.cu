@@ -15,7 +15,7 @@
 namespace fpx {
 namespace {
 
-__global__ void k_reset(Slot* slots, uint64_t n, Ctl* ctl) {
+__global__ void k_reset(Slot* slots, uint64_t n, Ctl* ctl, LiveSlot* live, uint32_t live_gen) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += stride) {
     Slot s;
@@ -25,7 +25,12 @@ __global__ void k_reset(Slot* slots, uint64_t n, Ctl* ctl) {
     s.pad = 0;
     slots[i] = s;
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) *ctl = Ctl{};
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    Ctl c{};
+    c.live = live;
+    c.live_gen = live_gen;
+    *ctl = c;
+  }
 }
 
 __device__ __forceinline__ void clear_slot(Slot* slots, uint64_t i) {
@@ -49,7 +54,13 @@ __global__ void k_reset_touched(const TableView tv, uint64_t slots) {
   }
 }
 
-__global__ void k_reset_ctl(Ctl* ctl) { *ctl = Ctl{}; }  // counters and padding (the whole block is copied to the host)
+// counters and padding (the whole block is copied to the host)
+__global__ void k_reset_ctl(Ctl* ctl, LiveSlot* live, uint32_t live_gen) {
+  Ctl c{};
+  c.live = live;
+  c.live_gen = live_gen;
+  *ctl = c;
+}
 
 __global__ void k_compact(const Slot* slots, uint64_t n, uint64_t* keys, uint64_t* counts, uint64_t* firsts,
                           unsigned long long* d_n) {
@@ -120,16 +131,17 @@ unsigned grid_for(uint64_t n) {
 
 }  // namespace
 
-cudaError_t launch_table_reset(const TableView& tv, uint64_t slots, cudaStream_t s) {
-  k_reset<<<grid_for(slots), 256, 0, s>>>(tv.slots, slots, tv.ctl);
+cudaError_t launch_table_reset(const TableView& tv, uint64_t slots, LiveSlot* live, uint32_t live_gen, cudaStream_t s) {
+  k_reset<<<grid_for(slots), 256, 0, s>>>(tv.slots, slots, tv.ctl, live, live_gen);
   return cudaGetLastError();
 }
 
-cudaError_t launch_table_reset_touched(const TableView& tv, uint64_t slots, cudaStream_t s) {
+cudaError_t launch_table_reset_touched(const TableView& tv, uint64_t slots, LiveSlot* live, uint32_t live_gen,
+                                      cudaStream_t s) {
   k_reset_touched<<<148 * 4, 256, 0, s>>>(tv, slots);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  k_reset_ctl<<<1, 1, 0, s>>>(tv.ctl);
+  k_reset_ctl<<<1, 1, 0, s>>>(tv.ctl, live, live_gen);
   return cudaGetLastError();
 }
 

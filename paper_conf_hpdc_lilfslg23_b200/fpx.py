@@ -86,6 +86,8 @@ _SIGS = {
 }
 EXPORTS = tuple(_SIGS)
 for _name, (_args, _res) in _SIGS.items():
+    if os.environ.get("FPX_LIB") and not hasattr(lib, _name):  # A/B against an older build (tuning only)
+        continue
     _f = getattr(lib, _name)
     _f.argtypes = _args
     _f.restype = _res

@@ -16,13 +16,16 @@ import numpy as np
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
-LIB = os.path.join(ROOT, "build", "libfpx_wt.so")
-CSRC = os.path.join(ROOT, "paper_conf_hpdc_lilfslg23_b200", "csrc")
+# WT_SRC: build the diagnostics library from another source tree (A/B against
+# an older commit's worktree); WT_TAG names the library
+SRC_ROOT = os.environ.get("WT_SRC", ROOT)
+LIB = os.path.join(ROOT, "build", f"libfpx_wt{os.environ.get('WT_TAG', '')}.so")
+CSRC = os.path.join(SRC_ROOT, "paper_conf_hpdc_lilfslg23_b200", "csrc")
 SRC = [os.path.join(CSRC, f) for f in ("fpx_api.cu", "fpx_scan_records.cu", "fpx_scan_tensor.cu", "fpx_table.cu")]
 
 os.makedirs(os.path.dirname(LIB), exist_ok=True)
 subprocess.run(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-Xcompiler",
-                "-fPIC,-O3", "-shared", "-I" + os.path.join(ROOT, "include"), "-DFPX_WARP_TIMES", *SRC, "-o", LIB],
+                "-fPIC,-O3", "-shared", "-I" + os.path.join(SRC_ROOT, "include"), "-DFPX_WARP_TIMES", *SRC, "-o", LIB],
                check=True)
 os.environ["FPX_LIB"] = LIB
 
