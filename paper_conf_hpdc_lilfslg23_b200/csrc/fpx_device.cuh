@@ -121,6 +121,17 @@ __device__ __forceinline__ void t_min(const TableView& tv, unsigned long long* a
   else atomicMin(a, v);
 }
 
+// Fire-and-forget reductions (no value returned: the issuing thread never
+// waits for the L2 round trip), same scopes as above.
+__device__ __forceinline__ void t_red_add(const TableView& tv, unsigned long long* a, unsigned long long v) {
+  if (tv.flags & TV_SHARED) asm volatile("red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(a), "l"(v) : "memory");
+  else asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(a), "l"(v) : "memory");
+}
+__device__ __forceinline__ void t_red_min(const TableView& tv, unsigned long long* a, unsigned long long v) {
+  if (tv.flags & TV_SHARED) asm volatile("red.relaxed.sys.global.min.u64 [%0], %1;" ::"l"(a), "l"(v) : "memory");
+  else asm volatile("red.relaxed.gpu.global.min.u64 [%0], %1;" ::"l"(a), "l"(v) : "memory");
+}
+
 // Insert-or-update.  Linear probing over the whole table: an event is only
 // dropped (and TABLE_FULL raised) when every slot holds another key.
 static __device__ __noinline__ void table_add(const TableView tv, unsigned long long key, unsigned long long cnt,
@@ -147,22 +158,22 @@ static __device__ __noinline__ void table_add(const TableView tv, unsigned long 
             *reinterpret_cast<volatile unsigned long long*>(&l->seq) = (tv.ctl->live_gen << 32) | (pos + 1ull);
           }
         } else {
-          t_add(tv, &tv.ctl->newlog_overflow, 1ull);
+          t_red_add(tv, &tv.ctl->newlog_overflow, 1ull);
         }
         k = key;
       }
     }
     if (k == key) {
-      t_add(tv, &s->count, cnt);
+      t_red_add(tv, &s->count, cnt);
       // `first` only decreases: a value already <= ours makes the min a no-op
       // (a fresh insert reads the empty slot's ~0 and always updates).  Skips
       // most of the atomics on hot slots: all-NaN storm S1 +20 % (A/B).
-      if (first < f_seen) t_min(tv, &s->first, first);
+      if (first < f_seen) t_red_min(tv, &s->first, first);
       return;
     }
     i = (i + 1) & tv.mask;
   }
-  t_add(tv, &tv.ctl->dropped_events, cnt);
+  t_red_add(tv, &tv.ctl->dropped_events, cnt);
 }
 
 // CTA-level pre-aggregation of table updates (dense exception storms): a
@@ -362,6 +373,11 @@ __device__ __forceinline__ void warp_flush_single(const TableView& tv, Pend& pen
 // Shared-memory address of a generic pointer into shared memory, and a
 // 128-bit shared load at such an address.
 __device__ __forceinline__ uint32_t sh_addr(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+__device__ __forceinline__ uint32_t sh_ld1(uint32_t addr) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+  return v;
+}
 __device__ __forceinline__ uint4 sh_ld4(uint32_t addr) {
   uint4 v;
   asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));

@@ -13,6 +13,10 @@
 #include "fpx_device.cuh"
 
 namespace fpx {
+#ifdef FPX_WARP_TIMES
+// diagnostics build: per warp, ns in the FLOW exact path's prologue / record loop / final flush
+__device__ unsigned long long g_phase_ns[3 * 148 * 32];
+#endif
 namespace rec {
 
 
@@ -293,6 +297,125 @@ __device__ __forceinline__ void count_staged(uint32_t sp, uint32_t dw, uint32_t 
       }
     }
   }
+}
+
+// One record evaluated from global memory (a recorded division, whose
+// sources the producer does not stage), out of line: rare, and kept out of
+// the lean FLOW path's register budget.
+template <int MODE>
+__device__ __noinline__ void flush_record_global(const RecDesc d, const uint32_t* __restrict__ lane_base, int lane,
+                                                 uint64_t gidx, const TableView tv, bool warm) {
+  PendingEvents<true> pend;
+  pend.warm = warm;
+  flush_record<MODE>(d, lane_base, lane, gidx, tv, pend, nullptr);
+  pend.flush(tv);
+}
+
+// The analyzer's exact path of a TMA tile (FLOW / FLOW_DETAIL, with warp
+// aggregation): record by record as the state of each lane depends on its
+// own destination and sources (Table 2), but lean: header fields
+// broadcast once, the planes read straight from the stage with LDS (lane l
+// reads its own word: conflict-free), the class / severity / kind rules
+// specialised per format, one code per lane, then Alg2's warp reduction per
+// distinct code (warp_flush_single).  Same result as exact_tile_records
+// (flow_code), ~4x fewer instructions per record: a NaN storm late in a
+// warp's work no longer keeps it busy long after the others (the C3 tail).
+// Records whose planes are not staged (recorded divisions, R1) take the
+// generic flush_record from global memory.
+template <int MODE, typename Needed>
+__device__ __forceinline__ void exact_tile_flow(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
+                                                const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
+                                                int lane, uint64_t gidx0, const TableView tv, bool warm,
+                                                Needed needed) {
+#ifdef FPX_WARP_TIMES
+  unsigned long long tph0;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tph0));
+#endif
+  uint4 h = make_uint4(0u, 0u, 0u, 0u);
+  if ((uint32_t)lane < k) h = hdr_tile[lane];
+  const bool ok = (uint32_t)lane < k && record_valid<MODE>(h, arena_planes);
+  const uint32_t mask = ok ? h.y : 0u;
+  const uint32_t c = (ok && mask != 0u) ? needed(h.z) : 0u;
+  uint32_t slot = c;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t t = __shfl_up_sync(FULL, slot, o);
+    if (lane >= o) slot += t;
+  }
+  slot -= c;
+#ifdef FPX_WARP_TIMES
+  unsigned long long tph1;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tph1));
+#endif
+  // per record, packed: stage slot (bits 0-7, 0xFF = not staged) | meta << 8
+  // (meta < 2^15 for a valid record)
+  const uint32_t packed = (c != 0u ? slot : 0xFFu) | (h.z << 8);
+  const uint32_t sbase = sh_addr(stage_lane);  // this lane's word of stage slot 0
+  PendingEvents<true> pend;
+  pend.warm = warm;
+  uint32_t todo = __ballot_sync(FULL, mask != 0u);
+  while (todo) {
+    const uint32_t j = (uint32_t)(__ffs(todo) - 1);
+    todo &= todo - 1u;
+    const uint32_t pk = __shfl_sync(FULL, packed, j), m = __shfl_sync(FULL, mask, j);
+    const uint32_t site = __shfl_sync(FULL, h.x, j);
+    const uint32_t meta = pk >> 8, sl = pk & 0xFFu;
+    if (sl == 0xFFu) {  // not staged: a recorded division (or no planes at all)
+      const RecDesc d{__shfl_sync(FULL, h.w, j), m, meta, site};
+      pend.flush(tv);  // keep the events in record order (PendingEvents merges neighbours)
+      flush_record_global<MODE>(d, lane_base, lane, gidx0 + j, tv, warm);
+      continue;
+    }
+    const uint32_t op = op_of(meta), fmt = fmt_of(meta), ns = nsrc_of(meta), dw = dwords_of(meta);
+    const uint32_t a = sbase + sl * 128u;  // this lane's word of the record's plane 0
+    // S: most severe source class (NaN > INF > SUB, R5), src: lowest index holding it (R21)
+    uint32_t sev = 0u, src = 0u, dcls = CLS_CLEAN;
+    if (fmt == FPX_FP64) {
+      for (uint32_t q = 0; q < ns; ++q) {
+        const uint32_t lo = sh_ld1(a + (dw + 2u * q) * 128u), hi = sh_ld1(a + (dw + 2u * q + 1u) * 128u);
+        const uint32_t cl = cls_fp64(lo, hi), sv = cl == CLS_CLEAN ? 0u : 4u - cl;
+        if (sv > sev) sev = sv, src = q;
+      }
+      if (dw != 0u) dcls = cls_fp64(sh_ld1(a), sh_ld1(a + 128u));
+    } else {
+      for (uint32_t q = 0; q < ns; ++q) {
+        const uint32_t cl = cls_fp32(sh_ld1(a + (dw + q) * 128u)), sv = cl == CLS_CLEAN ? 0u : 4u - cl;
+        if (sv > sev) sev = sv, src = q;
+      }
+      if (dw != 0u) dcls = cls_fp32(sh_ld1(a));
+    }
+    // D: Alg1's dispatch (dest_kind): RCP -> DIV0 iff NaN / INF; compares: none
+    int D = CODE_NONE;
+    if (op == FPX_OP_MUFU_RCP || op == FPX_OP_MUFU_RCP64H) D = (dcls == CLS_NAN || dcls == CLS_INF) ? FPX_DIV0 : CODE_NONE;
+    else if (!is_compare(op)) D = kind_of_cls(dcls);
+    // Table 2: GEN / PROP / KILL (the kind of a KILL is the source's, 4 - sev - 1)
+    int code = CODE_NONE;
+    if (D >= 0) code = ((sev ? FPX_PROP : FPX_GEN) << 2) | D;
+    else if (sev) code = (FPX_KILL << 2) | (int)(3u - sev);
+    if (MODE == FPX_MODE_FLOW_DETAIL && sev && code >= 0) {
+      const bool cf = op == FPX_OP_FSEL || op == FPX_OP_FSET || op == FPX_OP_FSETP || op == FPX_OP_FMNMX ||
+                      op == FPX_OP_DSETP;
+      code |= (int)((src + 1u) | (cf ? (uint32_t)FPX_DETAIL_CMP : 0u)) << 4;
+    }
+    if (((m >> lane) & 1u) == 0u) code = CODE_NONE;
+    warp_flush_single(tv, pend, code, site, fmt, gidx0 + j);
+  }
+#ifdef FPX_WARP_TIMES
+  unsigned long long tph2, tph3;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tph2));
+#endif
+  pend.flush(tv);
+#ifdef FPX_WARP_TIMES
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tph3));
+  if (lane == 0) {
+    const uint64_t gw = blockIdx.x * (uint64_t)(blockDim.x / 32) + threadIdx.x / 32;
+    if (gw < 148 * 32) {
+      g_phase_ns[3 * gw] += tph1 - tph0;
+      g_phase_ns[3 * gw + 1] += tph2 - tph1;
+      g_phase_ns[3 * gw + 2] += tph3 - tph2;
+    }
+  }
+#endif
 }
 
 // DEST-mode exact path of a TMA tile, transposed: lane j evaluates ALL lanes of

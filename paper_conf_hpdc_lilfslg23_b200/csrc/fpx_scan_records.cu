@@ -379,6 +379,10 @@ struct Sched {
 // start and end of the last record-scan launch, to measure load imbalance.
 constexpr int kMaxWarpTimes = 148 * 32;
 __device__ unsigned long long g_warp_t0[kMaxWarpTimes], g_warp_t1[kMaxWarpTimes];
+// per warp: hit tiles and time spent in the exact path (ns)
+__device__ unsigned long long g_warp_hits[kMaxWarpTimes], g_warp_exact_ns[kMaxWarpTimes];
+// per warp: tiles consumed, chunks claimed, ns waiting on the stage mbarrier
+__device__ unsigned long long g_warp_tiles[kMaxWarpTimes], g_warp_chunks[kMaxWarpTimes], g_warp_wait_ns[kMaxWarpTimes];
 #endif
 
 // The exact path of a hit tile (rec::exact_tile_hdr with this kernel's
@@ -395,10 +399,11 @@ __device__ __forceinline__ void exact_tile_ring(const uint4* __restrict__ hdr_ti
   });
 }
 // DEST: inlined (its transposed path fits the scan loop's registers: no
-// spill).  FLOW / FLOW_DETAIL: called through a function pointer -- a direct
-// call lets ptxas allocate caller and callee registers together and the
-// record-walking path's demands then spill the scan loop's live values (up
-// to 180 B per tile); an indirect call uses the ABI calling convention,
+// spill).  FLOW / FLOW_DETAIL (exact_tile_flow) and the no-aggregation
+// ablation (exact_tile_records): called through function pointers -- a
+// direct call lets ptxas allocate caller and callee registers together and
+// the record-walking path's demands then spill the scan loop's live values
+// (up to 230 B per tile); an indirect call uses the ABI calling convention,
 // whose saves and restores sit around the call, on the rare path only.
 template <int MODE>
 __device__ __noinline__ void exact_tile_ring_call(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
@@ -406,16 +411,23 @@ __device__ __noinline__ void exact_tile_ring_call(const uint4* __restrict__ hdr_
                                                   int lane, uint64_t gidx0, const TableView tv, bool warm) {
   exact_tile_ring<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, warm);
 }
+// The analyzer's lean exact path (rec::exact_tile_flow), out of line.
+template <int MODE>
+__device__ __noinline__ void exact_tile_flow_call(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
+                                                  const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
+                                                  int lane, uint64_t gidx0, const TableView tv, bool warm) {
+  exact_tile_flow<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, warm, [](uint32_t meta) {
+    bool f;
+    const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, f, f);
+    return fmt_of(meta) == FPX_FP64 ? 2u * ni : ni;
+  });
+}
 using ExactFn = void (*)(const uint4*, uint32_t, uint64_t, const uint32_t*, const uint32_t*, int, uint64_t,
                          const TableView, bool);
 template <int MODE>
 __device__ ExactFn g_exact_fn = exact_tile_ring_call<MODE>;
-#ifndef DESTCALL
-#define DESTCALL exact_tile_ring
-#endif
-#ifndef FLOWCALL
-#define FLOWCALL g_exact_fn
-#endif
+template <int MODE>
+__device__ ExactFn g_flow_fn = exact_tile_flow_call<MODE>;
 // the CTA table is used by a warp from its kWarmTiles-th hit tile on
 constexpr uint32_t kWarmTiles = 8;
 
@@ -447,7 +459,13 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     return;
   }
 #ifdef FPX_WARP_TIMES
-  if (lane == 0 && gw < kMaxWarpTimes) g_warp_t0[gw] = globaltimer_ns();
+  if (lane == 0 && gw < kMaxWarpTimes) {
+    g_warp_t0[gw] = globaltimer_ns();
+    g_warp_hits[gw] = 0;
+    g_warp_exact_ns[gw] = 0;
+    g_warp_tiles[gw] = g_warp_chunks[gw] = g_warp_wait_ns[gw] = 0;
+    g_phase_ns[3 * gw] = g_phase_ns[3 * gw + 1] = g_phase_ns[3 * gw + 2] = 0;
+  }
 #endif
   const uint64_t end = min(n, start + recs_per_warp);
   // dynamic tail (Sched): the chunk this warp takes after its current range,
@@ -478,6 +496,9 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       const uint32_t c = __shfl_sync(FULL, claim, 0);
       if (c < sch.nchunks) {
         cursor = c < sch.nbig ? sch.dyn0 + (uint64_t)c * sch.chunk : sch.dyn1 + (uint64_t)(c - sch.nbig) * TILE;
+#ifdef FPX_WARP_TIMES
+        if (lane == 0 && gw < kMaxWarpTimes) g_warp_chunks[gw] += 1;
+#endif
         rem = (uint32_t)min((uint64_t)(c < sch.nbig ? sch.chunk : TILE), n - cursor);
         if (lane == 0) claim = atomicAdd(sch.ctr, 1u);
       }
@@ -628,8 +649,17 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       cta_warp_done(tv, C::WARPS);
       break;
     }
+#ifdef FPX_WARP_TIMES
+    const uint64_t tw0 = globaltimer_ns();
+#endif
     mbar_wait(&sm.bar[s], (phase >> s) & 1u);
     phase ^= 1u << s;
+#ifdef FPX_WARP_TIMES
+    if (lane == 0 && gw < kMaxWarpTimes) {
+      g_warp_wait_ns[gw] += globaltimer_ns() - tw0;
+      g_warp_tiles[gw] += 1;
+    }
+#endif
 
     // ---- fast path over the staged planes (lane-quad layout) --------------
     const uint32_t ia = smem_u32(sm.items[s]), pa = smem_u32(sm.planes[s]);
@@ -654,20 +684,31 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       consume_list<FPX_BF16, false>(w, seg[6], seg[7], ia, pa, g, q);
       consume_list<FPX_BF16, true>(w, seg[7], seg[8], ia, pa, g, q);
     }
-    if (__any_sync(FULL, w.hit_wide() || (halves && w.hit_half())) || (mk & kForceBit) != 0u)
-    {
+    if (__any_sync(FULL, w.hit_wide() || (halves && w.hit_half())) || (mk & kForceBit) != 0u) {
       // hit tiles of this warp so far: kept in shared memory (the stage-0
       // descriptor's spare word), not in a register of the scan loop
       const uint32_t hits = sm.meta[0].pad[0];
       __syncwarp();
       if (lane == 0) sm.meta[0].pad[0] = hits + 1u;
       const bool warm = hits >= kWarmTiles;
+#ifdef FPX_WARP_TIMES
+      const uint64_t te0 = globaltimer_ns();
+#endif
       if (MODE == FPX_MODE_DEST)
-        DESTCALL<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base,
+        exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base,
                               sm.planes[s] + lane, lane, m.gidx0, tv, warm);
-      else
-        FLOWCALL<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
+      else if (!(tv.flags & FPX_OPT_NO_WARP_AGG))
+        g_flow_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
+                        lane, m.gidx0, tv, warm);
+      else  // the no-aggregation ablation's record-by-record path
+        g_exact_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
                          lane, m.gidx0, tv, warm);
+#ifdef FPX_WARP_TIMES
+      if (lane == 0 && gw < kMaxWarpTimes) {
+        g_warp_hits[gw] = hits + 1;
+        g_warp_exact_ns[gw] += globaltimer_ns() - te0;
+      }
+#endif
     }
   }
 }
@@ -965,6 +1006,27 @@ extern "C" __attribute__((visibility("default"))) int fpx_debug_warp_times(unsig
   if (n > fpx::kMaxWarpTimes) n = fpx::kMaxWarpTimes;
   if (cudaMemcpyFromSymbol(t0, fpx::g_warp_t0, n * sizeof(unsigned long long)) != cudaSuccess) return -1;
   if (cudaMemcpyFromSymbol(t1, fpx::g_warp_t1, n * sizeof(unsigned long long)) != cudaSuccess) return -1;
+  return n;
+}
+extern "C" __attribute__((visibility("default"))) int fpx_debug_warp_exact(unsigned long long* hits,
+                                                                            unsigned long long* ns, int n) {
+  if (n > fpx::kMaxWarpTimes) n = fpx::kMaxWarpTimes;
+  if (cudaMemcpyFromSymbol(hits, fpx::g_warp_hits, n * sizeof(unsigned long long)) != cudaSuccess) return -1;
+  if (cudaMemcpyFromSymbol(ns, fpx::g_warp_exact_ns, n * sizeof(unsigned long long)) != cudaSuccess) return -1;
+  return n;
+}
+extern "C" __attribute__((visibility("default"))) int fpx_debug_warp_counts(unsigned long long* tiles,
+                                                                             unsigned long long* chunks,
+                                                                             unsigned long long* wait_ns, int n) {
+  if (n > fpx::kMaxWarpTimes) n = fpx::kMaxWarpTimes;
+  if (cudaMemcpyFromSymbol(tiles, fpx::g_warp_tiles, n * sizeof(unsigned long long)) != cudaSuccess) return -1;
+  if (cudaMemcpyFromSymbol(chunks, fpx::g_warp_chunks, n * sizeof(unsigned long long)) != cudaSuccess) return -1;
+  if (cudaMemcpyFromSymbol(wait_ns, fpx::g_warp_wait_ns, n * sizeof(unsigned long long)) != cudaSuccess) return -1;
+  return n;
+}
+extern "C" __attribute__((visibility("default"))) int fpx_debug_warp_phases(unsigned long long* ph, int n) {
+  if (n > fpx::kMaxWarpTimes) n = fpx::kMaxWarpTimes;
+  if (cudaMemcpyFromSymbol(ph, fpx::g_phase_ns, 3 * n * sizeof(unsigned long long)) != cudaSuccess) return -1;
   return n;
 }
 #endif

@@ -186,5 +186,6 @@ def test_shared_tables_use_system_scope_atomics():
     (CUDA memory model: an atomic is atomic only within its scope)."""
     sass = subprocess.run(["cuobjdump", "-sass", LIB], capture_output=True, text=True, check=True).stdout
     for op in ("CAS", "ADD", "MIN"):
-        assert re.search(rf"ATOMG?\.E\.{op}\.64\.STRONG\.SYS", sass), op
-        assert re.search(rf"ATOMG?\.E\.{op}\.64\.STRONG\.GPU", sass), op
+        # ATOM (value returned) or REDG (fire-and-forget reduction)
+        assert re.search(rf"(ATOMG?|REDG)\.E\.{op}\.64\.STRONG\.SYS", sass), op
+        assert re.search(rf"(ATOMG?|REDG)\.E\.{op}\.64\.STRONG\.GPU", sass), op

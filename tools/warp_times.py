@@ -53,8 +53,21 @@ for name in sys.argv[1:] or ["c2", "c3", "c4a", "c5"]:
         n = wt.fpx_debug_warp_times(t0.ctypes.data, t1.ctypes.data, NW)
         live = (t0[:n] != 0) & (t1[:n] >= t0[:n])
         a, b = t0[:n][live].astype(np.int64), t1[:n][live].astype(np.int64)
+        hx = np.zeros(NW, dtype=np.uint64)
+        ex = np.zeros(NW, dtype=np.uint64)
+        if hasattr(wt, "fpx_debug_warp_exact"):
+            wt.fpx_debug_warp_exact(hx.ctypes.data, ex.ctypes.data, NW)
+        cnt3 = np.zeros((3, NW), dtype=np.uint64)
+        if hasattr(wt, "fpx_debug_warp_counts"):
+            wt.fpx_debug_warp_counts(cnt3[0].ctypes.data, cnt3[1].ctypes.data, cnt3[2].ctypes.data, NW)
+        ph = np.zeros(3 * NW, dtype=np.uint64)
+        if hasattr(wt, "fpx_debug_warp_phases"):
+            wt.fpx_debug_warp_phases(ph.ctypes.data, NW)
         if rep >= 2:
             spans.append((a, b))
+            last_exact = (hx[:n][live].astype(np.int64), ex[:n][live].astype(np.int64),
+                          ph.reshape(NW, 3)[:n][live].astype(np.int64), cnt3[:, :n][:, live].astype(np.int64),
+                          np.nonzero(live)[0])
         t0[:] = 0
         t1[:] = 0
     for a, b in spans[-2:]:
@@ -68,6 +81,24 @@ for name in sys.argv[1:] or ["c2", "c3", "c4a", "c5"]:
               f"{(a.max() - s0) / 1e3:.1f} us | end p10/p50/p90/max {ends[len(ends) // 10] / 1e3:.1f}/"
               f"{ends[len(ends) // 2] / 1e3:.1f}/{ends[9 * len(ends) // 10] / 1e3:.1f}/{ends[-1] / 1e3:.1f} us | "
               f"idle share {100 * idle:.1f} %", flush=True)
+    hits, ens, phs, c3, gws = last_exact
+    if c3.sum():
+        order = np.argsort(b - a)
+        med = order[len(order) // 2]
+        for tag, i in [("median", med)] + [("slow", i) for i in order[-6:]]:
+            print(f"  {tag:6s} warp {gws[i]:5d} (CTA {gws[i] // 20:3d}) dur {(b[i] - a[i]) / 1e3:6.1f} us start "
+                  f"{(a[i] - a.min()) / 1e3:5.1f} tiles {c3[0, i]:5d} chunks {c3[1, i]:3d} mbar wait "
+                  f"{c3[2, i] / 1e3:6.1f} us hits {hits[i]}", flush=True)
+    if phs.sum():
+        late = np.argsort(b - a)[-5:]
+        print("  FLOW exact phases (prologue / records / flush) of the 5 slowest warps: "
+              + ", ".join(f"{phs[i, 0] / 1e3:.1f}/{phs[i, 1] / 1e3:.1f}/{phs[i, 2] / 1e3:.1f} us" for i in late), flush=True)
+    if hits.sum():
+        late = np.argsort(b - a)[-5:]
+        print(f"  exact path: hit tiles total {hits.sum()}, per warp med/max {np.median(hits):.0f}/{hits.max()}, "
+              f"time per warp med/max {np.median(ens) / 1e3:.1f}/{ens.max() / 1e3:.1f} us; 5 slowest warps: "
+              + ", ".join(f"dur {(b[i] - a[i]) / 1e3:.1f} us hits {hits[i]} exact {ens[i] / 1e3:.1f} us" for i in late),
+              flush=True)
     h.close()
     del wl
     torch.cuda.empty_cache()
