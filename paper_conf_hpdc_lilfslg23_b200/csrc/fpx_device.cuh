@@ -206,11 +206,19 @@ struct CtaTable {
   __device__ __forceinline__ unsigned int* cnt() const { return reinterpret_cast<unsigned int*>(keys + CT_SLOTS); }
   __device__ __forceinline__ unsigned int* first() const { return cnt() + CT_SLOTS; }
   __device__ __forceinline__ bool on() const { return keys != nullptr; }
-  // The record-scan ring kernel keeps the table at the START of dynamic
-  // shared memory with its header in the last slot (key = base index,
-  // count = on, first = warps done), so the exact path finds it without any
-  // register held by the scan loop.
-  __device__ static CtaTable from_image(uint8_t* smem) {
+  // The record-scan ring kernel keeps the table at the END of its dynamic
+  // shared memory (image_at) with its header in the last slot (key = base
+  // index, count = on, first = warps done), so the exact path finds it from
+  // %dynamic_smem_size without any register held by the scan loop, and the
+  // rings keep their offsets.
+  __device__ static uint8_t* image_at() {
+    extern __shared__ __align__(128) uint8_t fpx_dyn_smem[];
+    uint32_t dyn;
+    asm("mov.u32 %0, %%dynamic_smem_size;" : "=r"(dyn));
+    return fpx_dyn_smem + dyn - bytes();
+  }
+  __device__ static CtaTable from_image() {
+    uint8_t* smem = image_at();
     const unsigned long long* k = reinterpret_cast<const unsigned long long*>(smem);
     const unsigned int* c = reinterpret_cast<const unsigned int*>(k + CT_SLOTS);
     return CtaTable{c[CT_USABLE] ? reinterpret_cast<unsigned long long*>(smem) : nullptr, k[CT_USABLE]};
@@ -266,10 +274,13 @@ struct CtaTable {
 // whose dynamic shared memory starts with a CtaTable image.
 static __device__ __noinline__ void emit_event(const TableView tv, unsigned long long key, uint32_t c,
                                               unsigned long long f, bool dense) {
-  extern __shared__ __align__(128) uint8_t fpx_dyn_smem[];
-  const CtaTable ct = CtaTable::from_image(fpx_dyn_smem);
+#if FPX_NO_CTA
+  table_add(tv, key, c, f);
+#else
+  const CtaTable ct = CtaTable::from_image();
   if (dense && ct.on()) ct.add(tv, key, c, f);
   else table_add(tv, key, c, f);
+#endif
 }
 
 // Called once by every warp of the ring kernel's CTA as it finishes
@@ -279,8 +290,7 @@ static __device__ __noinline__ void emit_event(const TableView tv, unsigned long
 // The arrival counter is the header slot's first-offset word.  Out of line,
 // like emit_event, so the scan loop keeps no register for it.
 static __device__ __noinline__ void cta_warp_done(const TableView tv, uint32_t nwarps) {
-  extern __shared__ __align__(128) uint8_t fpx_dyn_smem[];
-  const CtaTable ct = CtaTable::from_image(fpx_dyn_smem);
+  const CtaTable ct = CtaTable::from_image();
   if (!ct.on()) return;
   const uint32_t lane = threadIdx.x & 31u;
   __syncwarp();

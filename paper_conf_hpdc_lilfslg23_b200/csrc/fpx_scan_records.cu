@@ -139,7 +139,7 @@ constexpr uint32_t META_RESERVED = 0xFFFF80E0u;
 // CTA pre-aggregation table (fpx_device.cuh CtaTable)
 template <class C>
 constexpr size_t ring_smem() {
-  return CtaTable::bytes() + sizeof(WarpSmem<C>) * C::WARPS + DECODE_ENTRIES;
+  return sizeof(WarpSmem<C>) * C::WARPS + DECODE_ENTRIES + CtaTable::bytes();
 }
 
 // Header decode for the fast path, branch-free: validity (the contract of
@@ -308,6 +308,12 @@ __device__ __forceinline__ uint4 and4(uint4 a, uint4 b) { return make_uint4(a.x 
 #define FPX_CONSUME_UNROLL 1  // A/B on B200 (tools/ab.sh): 1 beats 2 and 4 by 2-5 %
 #endif
 constexpr int kConsumeUnroll = FPX_CONSUME_UNROLL;
+#ifndef FPX_NO_CTA
+#define FPX_NO_CTA 0
+#endif
+#ifndef FPX_BAD_SYS
+#define FPX_BAD_SYS 1
+#endif
 
 // Consume one item list with the lane-quad layout: thread (g = lane / 8,
 // q = lane % 8) reads words 4q..4q+3 (lanes 4q..4q+3 of the instrumented
@@ -438,10 +444,10 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
                    const TableView tv) {
   constexpr int STAGES = C::STAGES, PLANES = C::PLANES;
   static_assert(PLANES <= 64, "stage sizes keep the byte fields of the packed scan exact");
-  // dynamic shared memory: [CTA table][per-warp rings][decode table]
+  // dynamic shared memory: [per-warp rings][decode table][CTA table]
   extern __shared__ __align__(128) uint8_t fpx_dyn_smem[];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  uint8_t* rings = fpx_dyn_smem + CtaTable::bytes();
+  uint8_t* rings = fpx_dyn_smem;
   WarpSmem<C>& sm = reinterpret_cast<WarpSmem<C>*>(rings)[warp];
   uint8_t* lut = rings + sizeof(WarpSmem<C>) * C::WARPS;
   build_decode_table<MODE>(lut);
@@ -449,13 +455,17 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   // CtaTable; the exact path finds it through emit_event); off for the
   // no-aggregation ablation and for launches whose record offsets need more
   // than 32 bits
-  CtaTable{reinterpret_cast<unsigned long long*>(fpx_dyn_smem), base_index}
+#if !FPX_NO_CTA
+  CtaTable{reinterpret_cast<unsigned long long*>(CtaTable::image_at()), base_index}
       .init((tv.flags & FPX_OPT_NO_WARP_AGG) == 0u && n < (uint64_t)CT_NONE);
+#endif
   __syncthreads();
   const uint64_t gw = blockIdx.x * (uint64_t)C::WARPS + warp;
   const uint64_t start = gw * recs_per_warp;
   if (start >= n) {  // warp-uniform; no block-wide barriers below this line
+#if !FPX_NO_CTA
     cta_warp_done(tv, C::WARPS);
+#endif
     return;
   }
 #ifdef FPX_WARP_TIMES
@@ -544,7 +554,11 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     uint32_t force_any = 0u;
     if (__any_sync(FULL, in_tile && (!ok || force))) {
       const uint32_t bad = __ballot_sync(FULL, in_tile && !ok);
+#if FPX_BAD_SYS
       if (bad != 0u && lane == 0) atomicAdd_system(&tv.ctl->bad_records, (unsigned long long)__popc(bad));  // rare; system scope covers shared tables
+#else
+      if (bad != 0u && lane == 0) atomicAdd(&tv.ctl->bad_records, (unsigned long long)__popc(bad));
+#endif
       force_any = __ballot_sync(FULL, in_tile && force);
     }
     const uint32_t my_planes = ni << (fmt == FPX_FP64 ? 1u : 0u);  // = planes_of_items(c8)
@@ -646,7 +660,6 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
         atomicExch(sch.ctr, 0u);
         atomicExch(sch.ctr + 1, 0u);
       }
-      cta_warp_done(tv, C::WARPS);
       break;
     }
 #ifdef FPX_WARP_TIMES
@@ -711,6 +724,10 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 #endif
     }
   }
+  // out of the loop: the call's register conventions stay off the scan loop
+#if !FPX_NO_CTA
+  cta_warp_done(tv, C::WARPS);
+#endif
 }
 
 // Ring configurations compiled in; FPX_RING (environment, tuning only) picks

@@ -47,17 +47,21 @@ for cb in cubins:
         if ksub and ksub not in name:
             continue
         cur_in, cur_out = None, None
+        fresh = True  # the first //## line after an instruction is the innermost; later ones walk outwards
         ins = []
         for line in body.splitlines():
             m = re.match(r'\s*//## File "([^"]+)", line (\d+)(?: inlined at "([^"]+)", line (\d+))?', line)
             if m:
-                cur_in = (os.path.basename(m.group(1)), int(m.group(2)))
-                cur_out = (os.path.basename(m.group(3)), int(m.group(4))) if m.group(3) else cur_in
-                # nested inlining lists the outermost last on later lines; keep the last one seen
+                here = (os.path.basename(m.group(1)), int(m.group(2)))
+                if fresh:
+                    cur_in = here
+                    fresh = False
+                cur_out = (os.path.basename(m.group(3)), int(m.group(4))) if m.group(3) else here
                 continue
             m = re.match(r"\s*/\*([0-9a-f]{4,})\*/\s+(.*?);", line)
             if m:
                 ins.append((m.group(2).strip(), cur_in, cur_out))
+                fresh = True
         if len(ins) >= len(counts) * 0.9 and len(ins) <= len(counts) * 1.1:
             best = ins
             break
