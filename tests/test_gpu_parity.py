@@ -576,3 +576,22 @@ def test_fetch_new_truncated_windows_lose_nothing(fpx):
         d2, da2 = to_dev(h2, a2)
         h.scan_records(d2, da2)
         assert [int(e["site"]) for e in h.fetch_new(capacity=30)] == [500]
+
+
+@pytest.mark.parametrize("mode", [DEST, FLOW, FLOW_DETAIL])
+@pytest.mark.parametrize("dense", [1.0, 0.01])
+def test_storm_cta_preaggregation(fpx, mode, dense):
+    """Storms long enough for warps to warm up the CTA pre-aggregation table
+    (> 8 hit tiles per warp: 1.2e6 records on 2960 warps) and dense tiles
+    (>= 4 records with events): the table equals the oracle's, so the
+    shared-memory counts, the first-sighting inserts and the end-of-CTA flush
+    add up exactly; and equals the per-lane ablation."""
+    p = fpxgen.Params(seed=88, n_records=1_200_001, n_sites=200, recipe=fpxgen.RECIPE_STRESS, dense_nan=dense)
+    hdr, arena = fpxgen.generate_host(p)
+    base = 7 * 10**9
+    exp = oracle_scan(hdr, arena, base, mode).entries()
+    got, st, _ = gpu_scan(fpx, hdr, arena, base=base, mode=mode)
+    assert st == fpx.OK
+    assert_same(got, exp)
+    got2, _, _ = gpu_scan(fpx, hdr, arena, base=base, mode=mode, flags=fpx.OPT_NO_WARP_AGG)
+    assert_same(got2, exp)

@@ -44,6 +44,22 @@ hdr, arena, planes = fpxgen.generate_device(p)
 with fpx.Handle(0, table_log2_slots=5) as h:
     h.scan_records(hdr, arena, arena_planes=planes)
     h.fetch()
+# storms long enough for warm warps: the CTA pre-aggregation table (shared
+# atomics from 20 warps, end-of-CTA flush by the last warp), DEST and FLOW
+p = fpxgen.Params(seed=10, n_records=900_017, n_sites=40, recipe=fpxgen.RECIPE_STRESS, dense_nan=0.05)
+hdr, arena, planes = fpxgen.generate_device(p)
+for mode in (0, 1):
+    with fpx.Handle(0) as h:
+        h.scan_records(hdr, arena, mode=mode, arena_planes=planes)
+        h.fetch()
+# early notification ring (mapped host memory) and a shared (exported) table
+with fpx.Handle(0, flags=fpx.OPT_LIVE_NEW) as h:
+    h.export()
+    h.scan_records(hdr, arena, arena_planes=planes)
+    torch.cuda.synchronize()
+    h.poll_new()
+    h.fetch()
+del hdr, arena
 for dt in (torch.float32, torch.float64, torch.float16, torch.bfloat16):
     x = torch.randn(100_003, device=dev).to(dt)
     x[::997] = float("nan")
