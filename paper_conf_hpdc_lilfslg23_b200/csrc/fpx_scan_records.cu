@@ -368,7 +368,14 @@ __device__ __forceinline__ void consume_list(Witness& w, uint32_t b, uint32_t e,
 // counter pairs).  nchunks = 0: static ranges only.
 constexpr uint64_t kDynMinTiles = 16;  // dynamic tail only from 16 tiles per warp up
 constexpr uint32_t kDynChunk = 256;     // records per claimed chunk (8 tiles)
-constexpr int kStaticPct = 75;          // share of the trace in static ranges
+constexpr int kStaticPct = 75;          // share of the trace in static ranges (DEST)
+// FLOW / FLOW_DETAIL: a smaller static share.  Some SMs stream 1.4-1.6x
+// slower than the median (tools/warp_times.py: their warps finish 255 tiles
+// of a static range while others do 313 with 15 claimed chunks), and the
+// analyzer traces are short (C3: 0.65 ms), so a 75 % static range alone
+// outlasts the kernel on them; 45 %: C3 +1.3 %, C2 (DEST) would lose 0.7 %
+// (profiles/r2/ab_static.txt).
+constexpr int kStaticPctFlow = 45;
 constexpr uint32_t kTailTiles = 8;      // one-tile chunks at the end, per warp
 struct SchedCfg {
   int static_pct;
@@ -941,7 +948,7 @@ k_scan_records_ldg(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 struct Tuning {
   int ring = -1;  // -1: by trace size
   int sched = 1;
-  int static_pct = kStaticPct;
+  int static_pct = -1;  // -1: by mode (kStaticPct / kStaticPctFlow)
   uint32_t dyn_chunk = kDynChunk, tail_tiles = kTailTiles;
 };
 #ifdef FPX_TUNING
@@ -991,7 +998,8 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   int ring = tu.ring;
   if (ring < 0) ring = n <= (uint64_t)num_sms * 24 * TILE ? 3 : 1;
   if (tu.sched == 0) sched_ctr = nullptr;
-  const SchedCfg scfg{tu.static_pct, tu.dyn_chunk, tu.sched == 2 ? 0u : tu.tail_tiles};
+  const int static_pct = tu.static_pct >= 0 ? tu.static_pct : MODE == FPX_MODE_DEST ? kStaticPct : kStaticPctFlow;
+  const SchedCfg scfg{static_pct, tu.dyn_chunk, tu.sched == 2 ? 0u : tu.tail_tiles};
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   switch (ring) {
     case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, s);
