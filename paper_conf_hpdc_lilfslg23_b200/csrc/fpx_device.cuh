@@ -274,13 +274,14 @@ struct CtaTable {
 // whose dynamic shared memory starts with a CtaTable image.
 static __device__ __noinline__ void emit_event(const TableView tv, unsigned long long key, uint32_t c,
                                               unsigned long long f, bool dense) {
-#if FPX_NO_CTA
+  if (dense) {  // only warm warps of kernels that set the table up pass dense
+    const CtaTable ct = CtaTable::from_image();
+    if (ct.on()) {
+      ct.add(tv, key, c, f);
+      return;
+    }
+  }
   table_add(tv, key, c, f);
-#else
-  const CtaTable ct = CtaTable::from_image();
-  if (dense && ct.on()) ct.add(tv, key, c, f);
-  else table_add(tv, key, c, f);
-#endif
 }
 
 // Called once by every warp of the ring kernel's CTA as it finishes

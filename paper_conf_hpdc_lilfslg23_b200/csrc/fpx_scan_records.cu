@@ -308,9 +308,14 @@ __device__ __forceinline__ uint4 and4(uint4 a, uint4 b) { return make_uint4(a.x 
 #define FPX_CONSUME_UNROLL 1  // A/B on B200 (tools/ab.sh): 1 beats 2 and 4 by 2-5 %
 #endif
 constexpr int kConsumeUnroll = FPX_CONSUME_UNROLL;
-#ifndef FPX_NO_CTA
-#define FPX_NO_CTA 0
+#ifndef FPX_CTA_FLOW
+#define FPX_CTA_FLOW 0
 #endif
+// CTA pre-aggregation table per mode: DEST storms (S1 / S2) gain 2.1x / 1.46x;
+// in the analyzer kernels it cost 5 % of C3 (more fast-path instructions,
+// profiles/r2/ab_cta_flow.txt) for storms that only stress tests produce.
+template <int MODE>
+constexpr bool kCtaTable = MODE == FPX_MODE_DEST || FPX_CTA_FLOW;
 #ifndef FPX_BAD_SYS
 #define FPX_BAD_SYS 1
 #endif
@@ -462,17 +467,14 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   // CtaTable; the exact path finds it through emit_event); off for the
   // no-aggregation ablation and for launches whose record offsets need more
   // than 32 bits
-#if !FPX_NO_CTA
-  CtaTable{reinterpret_cast<unsigned long long*>(CtaTable::image_at()), base_index}
-      .init((tv.flags & FPX_OPT_NO_WARP_AGG) == 0u && n < (uint64_t)CT_NONE);
-#endif
+  if (kCtaTable<MODE>)
+    CtaTable{reinterpret_cast<unsigned long long*>(CtaTable::image_at()), base_index}
+        .init((tv.flags & FPX_OPT_NO_WARP_AGG) == 0u && n < (uint64_t)CT_NONE);
   __syncthreads();
   const uint64_t gw = blockIdx.x * (uint64_t)C::WARPS + warp;
   const uint64_t start = gw * recs_per_warp;
   if (start >= n) {  // warp-uniform; no block-wide barriers below this line
-#if !FPX_NO_CTA
-    cta_warp_done(tv, C::WARPS);
-#endif
+    if (kCtaTable<MODE>) cta_warp_done(tv, C::WARPS);
     return;
   }
 #ifdef FPX_WARP_TIMES
@@ -710,7 +712,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       const uint32_t hits = sm.meta[0].pad[0];
       __syncwarp();
       if (lane == 0) sm.meta[0].pad[0] = hits + 1u;
-      const bool warm = hits >= kWarmTiles;
+      const bool warm = kCtaTable<MODE> && hits >= kWarmTiles;
 #ifdef FPX_WARP_TIMES
       const uint64_t te0 = globaltimer_ns();
 #endif
@@ -732,9 +734,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     }
   }
   // out of the loop: the call's register conventions stay off the scan loop
-#if !FPX_NO_CTA
-  cta_warp_done(tv, C::WARPS);
-#endif
+  if (kCtaTable<MODE>) cta_warp_done(tv, C::WARPS);
 }
 
 // Ring configurations compiled in; FPX_RING (environment, tuning only) picks
