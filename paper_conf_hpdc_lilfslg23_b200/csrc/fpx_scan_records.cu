@@ -111,10 +111,10 @@ constexpr int NLISTS = 8;
 constexpr uint32_t kForceBit = 0x80000000u;
 struct StageMeta {
   uint32_t k;      // records in the tile (0 = no tile) | kForceBit
-  uint32_t pad0;
+  uint32_t tot;    // items in the tile (end of the last list)
   uint64_t gidx0;  // global index of the tile's first record
-  uint32_t tf;     // packed per-format item counts, full-mask lists (byte = format)
-  uint32_t tp;     // same, partial-mask lists
+  uint32_t sb;     // byte f: first item of format f's full-mask list
+  uint32_t sp;     // byte f: first item of format f's partial-mask list
   uint32_t pad[2];
 };
 
@@ -581,13 +581,14 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     fence_proxy_async_smem();
     // list l = 2 * fmt + partial; lists of lower formats come first
     const uint32_t tot_f = tf + tp;  // packed per-format item totals (<= 128 each)
+    // byte f of `below`: items of the formats before f (= the start of format
+    // f's full-mask list).  Every byte stays <= 40 (items <= planes), so the
+    // packed sums never carry.
+    const uint32_t below = (tot_f * 0x01010101u) << 8;
     const bool writes = in_tile && ni != 0u;
     uint32_t at = 0u;
     if (writes) {
-      // byte f of `below`: items of the formats before f; byte f of `own`:
-      // this record's place among format f's items (full list first).  Every
-      // byte stays <= 40 (items <= planes), so the packed sums never carry.
-      const uint32_t below = (tot_f * 0x01010101u) << 8;
+      // byte f of `own`: this record's place among format f's items (full list first)
       const uint32_t own = part ? tf + (sp - cp) : sf - cf;
       at = ((below + own) >> (8 * fmt)) & 0xFFu;
       sm.items[s][at] = make_uint2(slot, mask);
@@ -606,8 +607,9 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     if (lane == 0) {
       m.k = k | (force_any != 0u ? kForceBit : 0u);
       m.gidx0 = base_index + cursor;
-      m.tf = tf;
-      m.tp = tp;
+      m.sb = below;              // list starts, packed (consumer: one PRMT per bound)
+      m.sp = below + tf;
+      m.tot = (tot_f * 0x01010101u) >> 24;
     }
     // Copies.  Common case: every in-tile record with an arena footprint
     // needs all of it and the footprints are arena-adjacent in record order
@@ -685,26 +687,23 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 
     // ---- fast path over the staged planes (lane-quad layout) --------------
     const uint32_t ia = smem_u32(sm.items[s]), pa = smem_u32(sm.planes[s]);
-    // list l = items [seg[l], seg[l+1]); lists in order (fmt, full / partial)
-    const uint32_t tf = m.tf, tp = m.tp;
-    uint32_t seg[NLISTS + 1];
-    seg[0] = 0u;
-#pragma unroll
-    for (int f = 0; f < 4; ++f) {
-      seg[2 * f + 1] = seg[2 * f] + ((tf >> (8 * f)) & 0xFFu);
-      seg[2 * f + 2] = seg[2 * f + 1] + ((tp >> (8 * f)) & 0xFFu);
-    }
+    // lists in order (fmt, full / partial): format f's full list is
+    // [sb_f, sp_f), its partial list [sp_f, sb_{f+1}) (the last ends at tot)
+    const uint32_t sb = m.sb, sp = m.sp, tot = m.tot;
+    auto byte_of = [](uint32_t x, uint32_t f) { return __byte_perm(x, 0u, 0x4440u | f); };
     Witness w;
-    consume_list<FPX_FP32, false>(w, seg[0], seg[1], ia, pa, g, q);
-    consume_list<FPX_FP32, true>(w, seg[1], seg[2], ia, pa, g, q);
-    consume_list<FPX_FP64, false>(w, seg[2], seg[3], ia, pa, g, q);
-    consume_list<FPX_FP64, true>(w, seg[3], seg[4], ia, pa, g, q);
-    const bool halves = ((tf | tp) >> 16) != 0u;
+    const uint32_t s1 = byte_of(sb, 1), s2 = byte_of(sb, 2);
+    consume_list<FPX_FP32, false>(w, 0u, byte_of(sp, 0), ia, pa, g, q);
+    consume_list<FPX_FP32, true>(w, byte_of(sp, 0), s1, ia, pa, g, q);
+    consume_list<FPX_FP64, false>(w, s1, byte_of(sp, 1), ia, pa, g, q);
+    consume_list<FPX_FP64, true>(w, byte_of(sp, 1), s2, ia, pa, g, q);
+    const bool halves = s2 != tot;
     if (halves) {
-      consume_list<FPX_FP16, false>(w, seg[4], seg[5], ia, pa, g, q);
-      consume_list<FPX_FP16, true>(w, seg[5], seg[6], ia, pa, g, q);
-      consume_list<FPX_BF16, false>(w, seg[6], seg[7], ia, pa, g, q);
-      consume_list<FPX_BF16, true>(w, seg[7], seg[8], ia, pa, g, q);
+      const uint32_t s3 = byte_of(sb, 3);
+      consume_list<FPX_FP16, false>(w, s2, byte_of(sp, 2), ia, pa, g, q);
+      consume_list<FPX_FP16, true>(w, byte_of(sp, 2), s3, ia, pa, g, q);
+      consume_list<FPX_BF16, false>(w, s3, byte_of(sp, 3), ia, pa, g, q);
+      consume_list<FPX_BF16, true>(w, byte_of(sp, 3), tot, ia, pa, g, q);
     }
     if (__any_sync(FULL, w.hit_wide() || (halves && w.hit_half())) || (mk & kForceBit) != 0u) {
       // hit tiles of this warp so far: kept in shared memory (the stage-0
