@@ -459,3 +459,49 @@ def test_div_packed_halves_vs_ieee(fmt):
     t = oracle.Table()
     t.scan_records(h, a)
     assert table_dict(t.entries()) == {(1, fmt, NONE, INF): [1, 0]}
+
+
+# --------------------------------------------------------------------------
+# opclasses without a special rule (OTHER, MUFU_OTHER, HADD2 / HFMA2 / HMUL2,
+# HMMA): the destination class of every value (Alg1's non-RCP branch, R11,
+# R13), pinned per value against numpy's IEEE predicates, each format
+# ----------------------------------------------------------------------------
+@pytest.mark.parametrize("opclass", [0, 6, 15, 16, 17, 18])
+def test_plain_class_opclasses_vs_numpy(opclass):
+    rng = np.random.default_rng(opclass)
+    pools = {
+        FP32: [0x0, 0x80000000, 0x1, 0x7FFFFF, 0x800000, 0x7F800000, 0xFF800000, 0x7FC00000, 0x7F800001, 0x3F800000],
+        FP16: [0x0, 0x8000, 0x1, 0x3FF, 0x400, 0x7C00, 0xFC00, 0x7E00, 0x7C01, 0x3C00],
+        BF16: [0x0, 0x8000, 0x1, 0x7F, 0x80, 0x7F80, 0xFF80, 0x7FC0, 0x7F81, 0x3F80],
+    }
+    tr = Trace(seed=opclass)
+    exp = {}
+    for r, fmt in enumerate([FP32, FP16, BF16] * 4):
+        dw = 1 + r % 4 if opclass == 18 else 1
+        words = []
+        vals = []
+        for _ in range(dw):
+            if fmt == FP32:
+                v = rng.choice(pools[FP32], size=32).astype(np.uint64)
+                words.append(v)
+                vals.append(v)
+            else:
+                lo = rng.choice(pools[fmt], size=32).astype(np.uint64)
+                hi = rng.choice(pools[fmt], size=32).astype(np.uint64)
+                words.append(lo | (hi << np.uint64(16)))
+                vals += [lo, hi]
+        mask = int(rng.integers(1, 2**32))
+        tr.add(r, opclass, fmt, mask, words, [])
+        act = np.array([(mask >> l) & 1 for l in range(32)], dtype=bool)
+        for v in vals:
+            cls = np_class(fmt, v)
+            for c, k in ((C_NAN, NAN), (C_INF, INF), (C_SUB, SUB)):
+                cnt = int(((cls == c) & act).sum())
+                if cnt:
+                    e = exp.setdefault((r, fmt, NONE, k), [0, r])
+                    e[0] += cnt
+    hdr, arena = tr.arrays()
+    t = oracle.Table()
+    t.scan_records(hdr, arena)
+    assert t.bad_records == 0
+    assert table_dict(t.entries()) == exp
