@@ -284,6 +284,22 @@ static __device__ __noinline__ void emit_event(const TableView tv, unsigned long
   table_add(tv, key, c, f);
 }
 
+// A record's per-kind counts (16 bits per kind in cnt, kinds in `present`)
+// straight into the CTA table (warm warps, dense tiles of the transposed
+// DEST path); out of line like emit_event.
+static __device__ __noinline__ void emit_kinds_cta(const TableView tv, uint32_t site, uint32_t fmt, uint32_t present,
+                                                  unsigned long long cnt, unsigned long long f) {
+  const CtaTable ct = CtaTable::from_image();
+  while (present) {
+    const uint32_t kd = (uint32_t)(__ffs(present) - 1);
+    present &= present - 1u;
+    const unsigned long long key = make_key(site, fmt, kd);
+    const uint32_t c = (uint32_t)((cnt >> (16 * kd)) & 0xFFFFu);
+    if (ct.on()) ct.add(tv, key, c, f);
+    else table_add(tv, key, c, f);
+  }
+}
+
 // Called once by every warp of the ring kernel's CTA as it finishes
 // (warp-uniform).  The last one to arrive adds every slot's pending count
 // (with its min first index) to the device table: the other warps' shared

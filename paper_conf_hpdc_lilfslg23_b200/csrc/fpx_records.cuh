@@ -517,6 +517,13 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
   // and records run in parallel instead of one warp-wide round per kind (C1
   // +11 %).  A single kind (storms) updates right away (S2 -2 % otherwise).
   dense = warm && __popc(__ballot_sync(FULL, present != 0u)) >= kDenseEvents;
+  if (dense) {
+    // a warm warp in a storm: every record's per-kind counts go straight to
+    // the CTA table, whose shared-memory atomics merge equal keys -- no warp
+    // grouping (a segmented REDUX over many distinct peer groups is a loop)
+    if (present) emit_kinds_cta(tv, h.x, fmt, present, cnt, gidx0 + (uint64_t)lane);
+    return;
+  }
   uint32_t all = __reduce_or_sync(FULL, present), lead = 0u;
   if (__popc(all) == 1) {
     const uint32_t kd = (uint32_t)(__ffs(all) - 1);
