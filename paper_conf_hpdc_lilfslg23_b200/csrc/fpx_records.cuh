@@ -444,7 +444,7 @@ __device__ __forceinline__ void exact_tile_flow(const uint4* __restrict__ hdr_ti
 // Shared-memory reads are skewed (lane j reads instrumented lane (t + j) mod
 // 32 at step t) so the 32 lanes hit 32 different banks.  `h`, `c`, `slot`:
 // this lane's header, staged planes and stage slot.
-__device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t mask, uint32_t c, uint32_t slot,
+__device__ __forceinline__ bool exact_tile_transposed(const uint4 h, uint32_t mask, uint32_t c, uint32_t slot,
                                                       const uint32_t* __restrict__ arena, const uint32_t* stage,
                                                       int lane, uint64_t gidx0, const TableView& tv, bool warm) {
   // group leaders' updates go through the CTA table when there is one
@@ -522,7 +522,7 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
     // the CTA table, whose shared-memory atomics merge equal keys -- no warp
     // grouping (a segmented REDUX over many distinct peer groups is a loop)
     if (present) emit_kinds_cta(tv, h.x, fmt, present, cnt, gidx0 + (uint64_t)lane);
-    return;
+    return true;
   }
   uint32_t all = __reduce_or_sync(FULL, present), lead = 0u;
   if (__popc(all) == 1) {
@@ -534,7 +534,7 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
       const uint32_t sum = __reduce_add_sync(peers, (uint32_t)((cnt >> (16 * kd)) & 0xFFFFu));
       if ((uint32_t)lane == (uint32_t)(__ffs(peers) - 1)) emit(key, sum, gidx0 + (uint64_t)lane);
     }
-    return;
+    return false;
   }
   unsigned long long sums = 0ull;  // 16 bits per kind led by this lane
   while (all) {
@@ -557,6 +557,7 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
     lead &= lead - 1u;
     emit(make_key(h.x, fmt, kd), (uint32_t)((sums >> (16 * kd)) & 0xFFFFu), gidx0 + (uint64_t)lane);
   }
+  return false;
 }
 
 // Exact path of a hit TMA tile: DEST mode goes transposed
@@ -570,8 +571,9 @@ __device__ __forceinline__ void exact_tile_transposed(const uint4 h, uint32_t ma
 // (profiles/r1/ab_sched.txt).  A/B in profiles/r1/ab_producer.txt (ab9-ab16).
 // Table updates go through emit_event (the CTA pre-aggregation table, if the
 // kernel set one up, then the device table).
+// Returns whether the tile was dense (DEST transposed path, warm warp).
 template <int MODE, typename Needed>
-__device__ __forceinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
+__device__ __forceinline__ bool exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
                                             const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
                                             int lane, uint64_t gidx0, const TableView tv, bool warm, Needed needed) {
   if (MODE == FPX_MODE_DEST && !(tv.flags & FPX_OPT_NO_WARP_AGG)) {
@@ -586,10 +588,10 @@ __device__ __forceinline__ void exact_tile_hdr(const uint4* __restrict__ hdr_til
       const uint32_t t = __shfl_up_sync(FULL, slot, o);
       if (lane >= o) slot += t;
     }
-    exact_tile_transposed(h, mask, c, slot - c, lane_base - lane, stage_lane - lane, lane, gidx0, tv, warm);
-    return;
+    return exact_tile_transposed(h, mask, c, slot - c, lane_base - lane, stage_lane - lane, lane, gidx0, tv, warm);
   }
   exact_tile_records<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, warm, needed);
+  return false;
 }
 
 // Plane items of one record for the fast path, by list:

@@ -407,10 +407,10 @@ __device__ unsigned long long g_warp_tiles[kMaxWarpTimes], g_warp_chunks[kMaxWar
 // needed-plane count).  `warm`: this warp has met enough hit tiles for the
 // CTA pre-aggregation table to pay (a storm); dense tiles then go through it.
 template <int MODE>
-__device__ __forceinline__ void exact_tile_ring(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
+__device__ __forceinline__ bool exact_tile_ring(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
                                                 const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
                                                 int lane, uint64_t gidx0, const TableView tv, bool warm) {
-  exact_tile_hdr<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, warm, [](uint32_t meta) {
+  return exact_tile_hdr<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, warm, [](uint32_t meta) {
     bool f;
     const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, f, f);
     return fmt_of(meta) == FPX_FP64 ? 2u * ni : ni;
@@ -446,6 +446,8 @@ template <int MODE>
 __device__ ExactFn g_exact_fn = exact_tile_ring_call<MODE>;
 template <int MODE>
 __device__ ExactFn g_flow_fn = exact_tile_flow_call<MODE>;
+// storm mode (witnesses skipped) after this many dense exact tiles in a row
+constexpr uint32_t kStormTiles = 16;
 // the CTA table is used by a warp from its kWarmTiles-th hit tile on
 constexpr uint32_t kWarmTiles = 8;
 
@@ -653,7 +655,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     h = ld_stream4_if((uint32_t)lane < rem, hdr_lane + cursor);
   };
 
-  uint32_t phase = 0;  // bit s = parity to wait for on stage s
+  uint32_t phase = 0;      // bit s = parity to wait for on stage s
+  uint32_t storm_run = 0;  // dense exact tiles in a row (DEST storm mode)
 #pragma unroll 1
   for (int s = 0; s < STAGES - 1; ++s) produce(s);
 #pragma unroll 1
@@ -685,27 +688,34 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     }
 #endif
 
-    // ---- fast path over the staged planes (lane-quad layout) --------------
-    const uint32_t ia = smem_u32(sm.items[s]), pa = smem_u32(sm.planes[s]);
-    // lists in order (fmt, full / partial): format f's full list is
-    // [sb_f, sp_f), its partial list [sp_f, sb_{f+1}) (the last ends at tot)
-    const uint32_t sb = m.sb, sp = m.sp, tot = m.tot;
-    auto byte_of = [](uint32_t x, uint32_t f) { return __byte_perm(x, 0u, 0x4440u | f); };
-    Witness w;
-    const uint32_t s1 = byte_of(sb, 1), s2 = byte_of(sb, 2);
-    consume_list<FPX_FP32, false>(w, 0u, byte_of(sp, 0), ia, pa, g, q);
-    consume_list<FPX_FP32, true>(w, byte_of(sp, 0), s1, ia, pa, g, q);
-    consume_list<FPX_FP64, false>(w, s1, byte_of(sp, 1), ia, pa, g, q);
-    consume_list<FPX_FP64, true>(w, byte_of(sp, 1), s2, ia, pa, g, q);
-    const bool halves = s2 != tot;
-    if (halves) {
-      const uint32_t s3 = byte_of(sb, 3);
-      consume_list<FPX_FP16, false>(w, s2, byte_of(sp, 2), ia, pa, g, q);
-      consume_list<FPX_FP16, true>(w, byte_of(sp, 2), s3, ia, pa, g, q);
-      consume_list<FPX_BF16, false>(w, s3, byte_of(sp, 3), ia, pa, g, q);
-      consume_list<FPX_BF16, true>(w, byte_of(sp, 3), tot, ia, pa, g, q);
+    // Storm mode (DEST): after kStormTiles dense exact tiles in a row a warp
+    // skips the witnesses -- in a storm every tile is hit anyway -- and
+    // sends each tile straight to the exact path, until one is not dense.
+    bool hit = MODE == FPX_MODE_DEST && storm_run >= kStormTiles;
+    if (!hit) {
+      // ---- fast path over the staged planes (lane-quad layout) ------------
+      const uint32_t ia = smem_u32(sm.items[s]), pa = smem_u32(sm.planes[s]);
+      // lists in order (fmt, full / partial): format f's full list is
+      // [sb_f, sp_f), its partial list [sp_f, sb_{f+1}) (the last ends at tot)
+      const uint32_t sb = m.sb, sp = m.sp, tot = m.tot;
+      auto byte_of = [](uint32_t x, uint32_t f) { return __byte_perm(x, 0u, 0x4440u | f); };
+      Witness w;
+      const uint32_t s1 = byte_of(sb, 1), s2 = byte_of(sb, 2);
+      consume_list<FPX_FP32, false>(w, 0u, byte_of(sp, 0), ia, pa, g, q);
+      consume_list<FPX_FP32, true>(w, byte_of(sp, 0), s1, ia, pa, g, q);
+      consume_list<FPX_FP64, false>(w, s1, byte_of(sp, 1), ia, pa, g, q);
+      consume_list<FPX_FP64, true>(w, byte_of(sp, 1), s2, ia, pa, g, q);
+      const bool halves = s2 != tot;
+      if (halves) {
+        const uint32_t s3 = byte_of(sb, 3);
+        consume_list<FPX_FP16, false>(w, s2, byte_of(sp, 2), ia, pa, g, q);
+        consume_list<FPX_FP16, true>(w, byte_of(sp, 2), s3, ia, pa, g, q);
+        consume_list<FPX_BF16, false>(w, s3, byte_of(sp, 3), ia, pa, g, q);
+        consume_list<FPX_BF16, true>(w, byte_of(sp, 3), tot, ia, pa, g, q);
+      }
+      hit = __any_sync(FULL, w.hit_wide() || (halves && w.hit_half())) || (mk & kForceBit) != 0u;
     }
-    if (__any_sync(FULL, w.hit_wide() || (halves && w.hit_half())) || (mk & kForceBit) != 0u) {
+    if (hit) {
       // hit tiles of this warp so far: kept in shared memory (the stage-0
       // descriptor's spare word), not in a register of the scan loop
       const uint32_t hits = sm.meta[0].pad[0];
@@ -715,10 +725,11 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 #ifdef FPX_WARP_TIMES
       const uint64_t te0 = globaltimer_ns();
 #endif
-      if (MODE == FPX_MODE_DEST)
-        exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base,
-                              sm.planes[s] + lane, lane, m.gidx0, tv, warm);
-      else if (!(tv.flags & FPX_OPT_NO_WARP_AGG))
+      if (MODE == FPX_MODE_DEST) {
+        const bool dense = exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes,
+                                                 lane_base, sm.planes[s] + lane, lane, m.gidx0, tv, warm);
+        storm_run = dense ? min(storm_run + 1u, kStormTiles) : 0u;
+      } else if (!(tv.flags & FPX_OPT_NO_WARP_AGG))
         g_flow_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
                         lane, m.gidx0, tv, warm);
       else  // the no-aggregation ablation's record-by-record path
