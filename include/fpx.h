@@ -187,13 +187,18 @@ typedef struct {
 } fpx_options;
 
 /* Option flags.  FPX_OPT_LIVE_NEW enables early notification (fpx_poll_new
- * below).  The other two are ablations that compute the same table:
+ * below).  FPX_OPT_STORM always runs the record scan's storm kernel (a
+ * shared-memory pre-aggregation of the table updates per CTA; every tile
+ * straight to the exact path while a storm lasts); without it a DEST scan
+ * uses that kernel when the handle's previous scan sent at least a quarter
+ * of its tiles to the exact path — the table is the same either way.  The
+ * other two are ablations that compute the same table:
  * FPX_OPT_SCAN_LDG selects the register-staged LDG record-scan kernel instead
  * of the default TMA (cp.async.bulk) shared-memory ring.
  * FPX_OPT_NO_WARP_AGG turns off warp aggregation (Alg2) in the
  * record scans' exact path: every lane issues its own table updates, one per
  * distinct code it holds (SURVEY §8(d) stress ablation; record scans only). */
-enum { FPX_OPT_SCAN_LDG = 1, FPX_OPT_NO_WARP_AGG = 2, FPX_OPT_LIVE_NEW = 4 };
+enum { FPX_OPT_SCAN_LDG = 1, FPX_OPT_NO_WARP_AGG = 2, FPX_OPT_LIVE_NEW = 4, FPX_OPT_STORM = 8 };
 
 typedef struct {
   uint64_t bad_records;       /* records skipped by validation (sticky, cumulative) */

@@ -18,6 +18,7 @@ struct fpx_ctx {
   bool attached = false;  // table mapped from another process (fpx_open_attached)
   int num_sms = 148;
   uint32_t variant = 0;  // record-scan kernel: 0 TMA ring, 1 LDG (ablation)
+  bool force_storm = false;  // FPX_OPT_STORM: always the storm instantiation
   uint64_t slots = 0;
   TableView tv{};
   uint64_t newlog_cursor = 0;  // FETCH_NEW position
@@ -48,6 +49,11 @@ struct fpx_ctx {
   // early notification (FPX_OPT_LIVE_NEW): mapped pinned ring + poll cursor
   LiveSlot* h_live = nullptr;
   LiveSlot* d_live = nullptr;  // device view of h_live
+  // record-scan density feedback (storm kernel selection): mapped host struct
+  // + device accumulator
+  ScanFeedback* h_fb = nullptr;
+  ScanFeedback* d_fb_view = nullptr;
+  unsigned long long* d_fb_acc = nullptr;
   uint32_t live_gen = 1;       // bumped at every reset
   uint64_t live_cursor = 0;
 };
@@ -73,6 +79,23 @@ bool alloc_sched(fpx_ctx* h) {
     return false;
   }
   return cudaMemsetAsync(h->d_sched, 0, b, nullptr) == cudaSuccess;
+}
+
+// The record scan's density feedback (fpx_internal.h ScanFeedback).
+bool alloc_feedback(fpx_ctx* h) {
+  if (cudaHostAlloc(&h->h_fb, sizeof(ScanFeedback), cudaHostAllocMapped) != cudaSuccess) {
+    cudaGetLastError();
+    h->h_fb = nullptr;
+    return false;
+  }
+  std::memset(h->h_fb, 0, sizeof(ScanFeedback));
+  if (cudaHostGetDevicePointer(&h->d_fb_view, h->h_fb, 0) != cudaSuccess ||
+      cudaMalloc(&h->d_fb_acc, sizeof(unsigned long long)) != cudaSuccess ||
+      cudaMemsetAsync(h->d_fb_acc, 0, sizeof(unsigned long long), nullptr) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return true;
 }
 
 #define CK(x)                                                  \
@@ -208,7 +231,8 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   *out = nullptr;
   fpx_options o{};
   if (opt) o = *opt;
-  if ((o.flags & ~(uint32_t)(FPX_OPT_SCAN_LDG | FPX_OPT_NO_WARP_AGG | FPX_OPT_LIVE_NEW)) != 0) return FPX_ERR_INVALID;
+  if ((o.flags & ~(uint32_t)(FPX_OPT_SCAN_LDG | FPX_OPT_NO_WARP_AGG | FPX_OPT_LIVE_NEW | FPX_OPT_STORM)) != 0)
+    return FPX_ERR_INVALID;
   if (o.table_log2_slots == 0) o.table_log2_slots = 20;
   if (o.table_log2_slots < 4 || o.table_log2_slots > 30) return FPX_ERR_INVALID;
   int ndev = 0;
@@ -220,6 +244,7 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   if (!h) return FPX_ERR_NOMEM;
   h->device = device;
   h->variant = (o.flags & FPX_OPT_SCAN_LDG) ? 1u : 0u;
+  h->force_storm = (o.flags & FPX_OPT_STORM) != 0;
   h->slots = 1ull << o.table_log2_slots;
   // every failure below releases what was built so far through fpx_close
   // (which tolerates the members still null)
@@ -252,7 +277,7 @@ fpx_status fpx_open(int device, const fpx_options* opt, fpx_handle* out) {
   }
   e = launch_table_reset(h->tv, h->slots, h->d_live, h->live_gen, nullptr);
   if (e != cudaSuccess) return fail(cuda_err(e, "launch_table_reset"));
-  if (!alloc_sched(h)) return fail(FPX_ERR_NOMEM);
+  if (!alloc_sched(h) || !alloc_feedback(h)) return fail(FPX_ERR_NOMEM);
   e = cudaStreamSynchronize(nullptr);
   if (e != cudaSuccess) return fail(cuda_err(e, "cudaStreamSynchronize"));
   *out = h;
@@ -271,8 +296,18 @@ fpx_status fpx_scan_records(fpx_handle h, const fpx_rec_hdr* d_hdr, uint64_t n_r
   if (!g.ok) return cuda_err(cudaGetLastError(), "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   unsigned int* sched = h->d_sched + 2 * (h->sched_seq++ % kSchedSlots);
+  // storm kernel when forced, or when the handle's last published DEST launch
+  // sent at least a quarter of its tiles (~records / 32) to the exact path;
+  // read without synchronising (the value may be a launch or two old)
+  bool storm = h->force_storm;
+  if (!storm && h->h_fb != nullptr) {
+    const volatile ScanFeedback* fb = h->h_fb;
+    const uint64_t recs = fb->records, hits = fb->hit_tiles;
+    storm = recs != 0 && hits * 128u >= recs;
+  }
+  const FeedbackPtrs fbp{mode == FPX_MODE_DEST ? h->d_fb_acc : nullptr, h->d_fb_view};
   CK(launch_scan_records(d_hdr, n_records, d_arena, arena_planes, base_index, mode, h->tv, h->num_sms, h->variant,
-                         sched, s));
+                         sched, fbp, storm, s));
   h->last_stream = s;
   return FPX_OK;
 }
@@ -621,7 +656,7 @@ fpx_status fpx_open_attached(int device, const fpx_ipc_table* t, fpx_handle* out
     delete h;
     return FPX_ERR_NOMEM;
   }
-  if (!alloc_sched(h)) {
+  if (!alloc_sched(h) || !alloc_feedback(h)) {
     fpx_close(h);
     return FPX_ERR_NOMEM;
   }
@@ -652,6 +687,8 @@ fpx_status fpx_close(fpx_handle h) {
     }
     cudaFreeHost(h->h_ctl);
     if (h->h_live) cudaFreeHost(h->h_live);
+    if (h->h_fb) cudaFreeHost(h->h_fb);
+    if (h->d_fb_acc) cudaFree(h->d_fb_acc);
     if (h->h_list) cudaFreeHost(h->h_list);
     if (h->d_list) cudaFree(h->d_list);
     if (h->list_copied) cudaEventDestroy(h->list_copied);

@@ -81,14 +81,29 @@ struct alignas(16) ListEntry {
 };
 static_assert(sizeof(ListEntry) == 64, "list entry is 64 B");
 
+// Density feedback of the record scan (mapped pinned host memory, one per
+// handle): the last warp of a launch with a dynamic tail writes the launch's
+// hit tiles (tiles that took the exact path) and record count; the launcher
+// reads it, without synchronising, to pick the storm kernel for the next
+// launch of the handle.
+struct ScanFeedback {
+  unsigned long long hit_tiles;
+  unsigned long long records;
+};
+struct FeedbackPtrs {
+  unsigned long long* dev;  // device accumulator (zeroed again by the last warp), or nullptr
+  ScanFeedback* host;       // device view of the mapped host struct
+};
+
 // ---- launchers (fpx_scan_records.cu, fpx_scan_tensor.cu, fpx_table.cu) --------------------------------
 // variant 0 = TMA ring (default), 1 = register-staged LDG (FPX_OPT_SCAN_LDG ablation).
 // sched_ctr: two zeroed u32 counters of the TMA kernel's dynamic tail, left
 // zeroed again when the launch completes (nullptr: static ranges only).
+// storm: launch the DEST storm instantiation (CTA pre-aggregation, storm mode).
 cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena,
                                 uint64_t arena_planes, uint64_t base_index, uint32_t mode,
                                 const TableView& tv, int num_sms, uint32_t variant, unsigned int* sched_ctr,
-                                cudaStream_t s);
+                                const FeedbackPtrs& fbp, bool storm, cudaStream_t s);
 cudaError_t launch_scan_tensor(const void* d_ptr, uint64_t n_elems, uint32_t fmt, uint32_t site,
                                uint64_t base_index, const TableView& tv, int num_sms, cudaStream_t s);
 cudaError_t launch_scan_tensor_list(const ListEntry* d_entries, uint32_t n, uint64_t total_vec,

@@ -311,11 +311,13 @@ constexpr int kConsumeUnroll = FPX_CONSUME_UNROLL;
 #ifndef FPX_CTA_FLOW
 #define FPX_CTA_FLOW 0
 #endif
-// CTA pre-aggregation table per mode: DEST storms (S1 / S2) gain 2.1x / 1.46x;
-// in the analyzer kernels it cost 5 % of C3 (more fast-path instructions,
-// profiles/r2/ab_cta_flow.txt) for storms that only stress tests produce.
-template <int MODE>
-constexpr bool kCtaTable = MODE == FPX_MODE_DEST || FPX_CTA_FLOW;
+// The storm machinery (CTA pre-aggregation table, storm mode) lives in a
+// separate DEST kernel instantiation (STORM = true) that the launcher picks
+// when the handle's previous launch found a storm (ScanFeedback): it costs
+// the sparse fast path 1-2 % of its instructions (C2 / C5), and gains 2.7-3x
+// on storms.  The analyzer kernels never use it (it cost 5 % of C3).
+template <int MODE, bool STORM>
+constexpr bool kCtaTable = STORM && (MODE == FPX_MODE_DEST || FPX_CTA_FLOW);
 #ifndef FPX_BAD_SYS
 #define FPX_BAD_SYS 1
 #endif
@@ -390,6 +392,10 @@ struct Sched {
   unsigned int* ctr;
   uint64_t dyn0, dyn1;
   uint32_t chunk, nbig, nchunks, nwarps;
+  // density feedback: every warp adds its hit tiles to *fb_dev; the last warp
+  // out publishes the launch's total to mapped host memory (fb_host)
+  unsigned long long* fb_dev;
+  ScanFeedback* fb_host;
 };
 
 #ifdef FPX_WARP_TIMES
@@ -451,7 +457,7 @@ constexpr uint32_t kStormTiles = 16;
 // the CTA table is used by a warp from its kWarmTiles-th hit tile on
 constexpr uint32_t kWarmTiles = 8;
 
-template <int MODE, class C>
+template <int MODE, class C, bool STORM>
 __global__ void __launch_bounds__(C::WARPS * 32, 1)
 k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __restrict__ arena,
                    uint64_t arena_planes, uint64_t base_index, uint64_t recs_per_warp, const Sched sch,
@@ -469,14 +475,14 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   // CtaTable; the exact path finds it through emit_event); off for the
   // no-aggregation ablation and for launches whose record offsets need more
   // than 32 bits
-  if (kCtaTable<MODE>)
+  if (kCtaTable<MODE, STORM>)
     CtaTable{reinterpret_cast<unsigned long long*>(CtaTable::image_at()), base_index}
         .init((tv.flags & FPX_OPT_NO_WARP_AGG) == 0u && n < (uint64_t)CT_NONE);
   __syncthreads();
   const uint64_t gw = blockIdx.x * (uint64_t)C::WARPS + warp;
   const uint64_t start = gw * recs_per_warp;
   if (start >= n) {  // warp-uniform; no block-wide barriers below this line
-    if (kCtaTable<MODE>) cta_warp_done(tv, C::WARPS);
+    if (kCtaTable<MODE, STORM>) cta_warp_done(tv, C::WARPS);
     return;
   }
 #ifdef FPX_WARP_TIMES
@@ -503,6 +509,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     for (int s = 0; s < STAGES; ++s) mbar_init(&sm.bar[s], 1);
     mbar_init_fence();
     sm.meta[0].pad[0] = 0u;  // hit tiles of this warp (exact path, CTA-table warm-up)
+    sm.meta[0].pad[1] = 0u;  // dense exact tiles in a row (storm mode)
   }
   __syncwarp();
 
@@ -655,8 +662,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     h = ld_stream4_if((uint32_t)lane < rem, hdr_lane + cursor);
   };
 
-  uint32_t phase = 0;      // bit s = parity to wait for on stage s
-  uint32_t storm_run = 0;  // dense exact tiles in a row (DEST storm mode)
+  uint32_t phase = 0;  // bit s = parity to wait for on stage s
 #pragma unroll 1
   for (int s = 0; s < STAGES - 1; ++s) produce(s);
 #pragma unroll 1
@@ -669,10 +675,22 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 #ifdef FPX_WARP_TIMES
       if (lane == 0 && gw < kMaxWarpTimes) g_warp_t1[gw] = globaltimer_ns();
 #endif
-      // the last warp out re-arms the launch's chunk counters for reuse
-      if (sch.nchunks != 0u && lane == 0 && atomicAdd(sch.ctr + 1, 1u) == sch.nwarps - 1u) {
-        atomicExch(sch.ctr, 0u);
-        atomicExch(sch.ctr + 1, 0u);
+      // the last warp out re-arms the launch's chunk counters for reuse and
+      // publishes the launch's hit tiles (density feedback for the launcher)
+      if (sch.nchunks != 0u && lane == 0) {
+        const uint32_t my_hits = sm.meta[0].pad[0];
+        if (my_hits != 0u && sch.fb_dev != nullptr) atomicAdd(sch.fb_dev, (unsigned long long)my_hits);
+        __threadfence();
+        if (atomicAdd(sch.ctr + 1, 1u) == sch.nwarps - 1u) {
+          atomicExch(sch.ctr, 0u);
+          atomicExch(sch.ctr + 1, 0u);
+          if (sch.fb_dev != nullptr) {
+            const unsigned long long total = atomicExch(sch.fb_dev, 0ull);
+            volatile ScanFeedback* fb = sch.fb_host;
+            fb->hit_tiles = total;
+            fb->records = n;
+          }
+        }
       }
       break;
     }
@@ -691,7 +709,10 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     // Storm mode (DEST): after kStormTiles dense exact tiles in a row a warp
     // skips the witnesses -- in a storm every tile is hit anyway -- and
     // sends each tile straight to the exact path, until one is not dense.
-    bool hit = MODE == FPX_MODE_DEST && storm_run >= kStormTiles;
+    // (the run length lives in the stage-0 descriptor's spare word: a register
+    // held across the loop cost S2 6 %, profiles/r2/ab_storm_state.txt)
+    const uint32_t storm_run = kCtaTable<MODE, STORM> ? sm.meta[0].pad[1] : 0u;
+    bool hit = kCtaTable<MODE, STORM> && storm_run >= kStormTiles;
     if (!hit) {
       // ---- fast path over the staged planes (lane-quad layout) ------------
       const uint32_t ia = smem_u32(sm.items[s]), pa = smem_u32(sm.planes[s]);
@@ -721,14 +742,14 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       const uint32_t hits = sm.meta[0].pad[0];
       __syncwarp();
       if (lane == 0) sm.meta[0].pad[0] = hits + 1u;
-      const bool warm = kCtaTable<MODE> && hits >= kWarmTiles;
+      const bool warm = kCtaTable<MODE, STORM> && hits >= kWarmTiles;
 #ifdef FPX_WARP_TIMES
       const uint64_t te0 = globaltimer_ns();
 #endif
       if (MODE == FPX_MODE_DEST) {
         const bool dense = exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes,
                                                  lane_base, sm.planes[s] + lane, lane, m.gidx0, tv, warm);
-        storm_run = dense ? min(storm_run + 1u, kStormTiles) : 0u;
+        if (kCtaTable<MODE, STORM> && lane == 0) sm.meta[0].pad[1] = dense ? min(storm_run + 1u, kStormTiles) : 0u;
       } else if (!(tv.flags & FPX_OPT_NO_WARP_AGG))
         g_flow_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
                         lane, m.gidx0, tv, warm);
@@ -744,7 +765,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     }
   }
   // out of the loop: the call's register conventions stay off the scan loop
-  if (kCtaTable<MODE>) cta_warp_done(tv, C::WARPS);
+  if (kCtaTable<MODE, STORM>) cta_warp_done(tv, C::WARPS);
 }
 
 // Ring configurations compiled in; FPX_RING (environment, tuning only) picks
@@ -759,10 +780,10 @@ static_assert(sizeof(WarpSmem<Ring2>) % 128 == 0 && ring_smem<Ring0>() <= 227 * 
 
 constexpr int kMaxDevices = 64;
 
-template <int MODE, class C>
+template <int MODE, class C, bool STORM>
 cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uint64_t arena_planes, uint64_t base_index,
                         const TableView& tv, int num_sms, unsigned int* sched_ctr, const SchedCfg& scfg,
-                        cudaStream_t s) {
+                        const FeedbackPtrs& fbp, cudaStream_t s) {
   // the shared-memory opt-in, once per device and kernel instantiation;
   // handles may live on different host threads
   static std::once_flag once[kMaxDevices];
@@ -771,7 +792,7 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
   auto set_attr = [] {
-    return cudaFuncSetAttribute(k_scan_records_tma<MODE, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    return cudaFuncSetAttribute(k_scan_records_tma<MODE, C, STORM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)ring_smem<C>());
   };
   if (dev < kMaxDevices) {
@@ -784,7 +805,7 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
   // one CTA per SM; each warp a contiguous range of records (whole tiles of 32
   // where possible, so that ranges stay 512-B aligned in the header array)
   const uint64_t warps = (uint64_t)num_sms * C::WARPS;
-  Sched sch{sched_ctr, n, n, 0u, 0u, 0u, 0u};
+  Sched sch{sched_ctr, n, n, 0u, 0u, 0u, 0u, fbp.dev, fbp.host};
   uint64_t per, blocks;
   if (sched_ctr != nullptr && n >= warps * TILE * kDynMinTiles) {
     // static ranges: 3/4 of the trace in whole tiles; the rest in chunks
@@ -806,7 +827,7 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
     blocks = ((n + per - 1) / per + C::WARPS - 1) / C::WARPS;
   }
   if (per >= (1ull << 31)) return cudaErrorInvalidValue;  // the kernel counts a warp's records in 32 bits
-  k_scan_records_tma<MODE, C><<<(unsigned)blocks, C::WARPS * 32, ring_smem<C>(), s>>>(hdr, n, arena, arena_planes,
+  k_scan_records_tma<MODE, C, STORM><<<(unsigned)blocks, C::WARPS * 32, ring_smem<C>(), s>>>(hdr, n, arena, arena_planes,
                                                                                       base_index, per, sch, tv);
   return cudaGetLastError();
 }
@@ -985,7 +1006,7 @@ const Tuning& tuning() {
 template <int MODE>
 cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena, uint64_t arena_planes,
                              uint64_t base_index, const TableView& tv, int num_sms, uint32_t variant,
-                             unsigned int* sched_ctr, cudaStream_t s) {
+                             unsigned int* sched_ctr, const FeedbackPtrs& fbp, bool storm, cudaStream_t s) {
   if (variant == 1u) {
     const uint64_t tiles = (n + TILE - 1) / TILE;
     uint64_t blocks = (tiles + LDG_WARPS - 1) / LDG_WARPS;
@@ -1011,11 +1032,21 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   const int static_pct = tu.static_pct >= 0 ? tu.static_pct : MODE == FPX_MODE_DEST ? kStaticPct : kStaticPctFlow;
   const SchedCfg scfg{static_pct, tu.dyn_chunk, tu.sched == 2 ? 0u : tu.tail_tiles};
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
+  if constexpr (MODE == FPX_MODE_DEST) {
+    if (storm) {  // the storm instantiation (CTA table, storm mode)
+    switch (ring) {
+      case 1: return launch_ring<MODE, Ring1, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
+      case 2: return launch_ring<MODE, Ring2, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
+      case 3: return launch_ring<MODE, Ring3, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
+      default: return launch_ring<MODE, Ring0, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
+      }
+    }
+  }
   switch (ring) {
-    case 1: return launch_ring<MODE, Ring1>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, s);
-    case 2: return launch_ring<MODE, Ring2>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, s);
-    case 3: return launch_ring<MODE, Ring3>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, s);
-    default: return launch_ring<MODE, Ring0>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, s);
+    case 1: return launch_ring<MODE, Ring1, false>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
+    case 2: return launch_ring<MODE, Ring2, false>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
+    case 3: return launch_ring<MODE, Ring3, false>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
+    default: return launch_ring<MODE, Ring0, false>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
   }
 }
 
@@ -1023,12 +1054,15 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
 
 cudaError_t launch_scan_records(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_t* d_arena, uint64_t arena_planes,
                                 uint64_t base_index, uint32_t mode, const TableView& tv, int num_sms, uint32_t variant,
-                                unsigned int* sched_ctr, cudaStream_t s) {
+                                unsigned int* sched_ctr, const FeedbackPtrs& fbp, bool storm, cudaStream_t s) {
   if (mode == FPX_MODE_DEST)
-    return launch_records_t<FPX_MODE_DEST>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, sched_ctr, s);
+    return launch_records_t<FPX_MODE_DEST>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, sched_ctr,
+                                           fbp, storm, s);
   if (mode == FPX_MODE_FLOW)
-    return launch_records_t<FPX_MODE_FLOW>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, sched_ctr, s);
-  return launch_records_t<FPX_MODE_FLOW_DETAIL>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, sched_ctr, s);
+    return launch_records_t<FPX_MODE_FLOW>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant, sched_ctr,
+                                           fbp, false, s);
+  return launch_records_t<FPX_MODE_FLOW_DETAIL>(d_hdr, n, d_arena, arena_planes, base_index, tv, num_sms, variant,
+                                                sched_ctr, fbp, false, s);
 }
 
 }  // namespace fpx

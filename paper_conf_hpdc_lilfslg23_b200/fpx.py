@@ -31,6 +31,7 @@ FETCH_ALL, FETCH_NEW = 0, 1
 OPT_SCAN_LDG = 1
 OPT_NO_WARP_AGG = 2  # ablation: no warp aggregation in the record scans' exact path
 OPT_LIVE_NEW = 4  # early notification: new keys published to mapped host memory (fpx_poll_new)
+OPT_STORM = 8  # always the record scan's storm kernel (else chosen from the previous scan's density)
 KEY_EMPTY = 0xFFFFFFFFFFFFFFFF
 
 ENTRY_DTYPE = np.dtype(

@@ -58,7 +58,7 @@ def test_binding_names_match_header():
         if short.startswith("ERR_") or short in ("OK",):
             assert getattr(fpx, short) == val, name
         elif short in ("FP32", "FP64", "FP16", "BF16", "NAN", "INF", "SUB", "DIV0", "GEN", "PROP", "KILL",
-                       "FLOW_NONE", "MODE_DEST", "MODE_FLOW", "FETCH_ALL", "FETCH_NEW", "OPT_SCAN_LDG", "OPT_NO_WARP_AGG", "OPT_LIVE_NEW"):
+                       "FLOW_NONE", "MODE_DEST", "MODE_FLOW", "FETCH_ALL", "FETCH_NEW", "OPT_SCAN_LDG", "OPT_NO_WARP_AGG", "OPT_LIVE_NEW", "OPT_STORM"):
             assert getattr(fpx, short) == val, name
     assert e["FPX_OP_COUNT"] == 20 and e["FPX_OP_DIV"] == 19 and e["FPX_OP_MUFU_RCP64H"] == 5
 

@@ -582,16 +582,35 @@ def test_fetch_new_truncated_windows_lose_nothing(fpx):
 @pytest.mark.parametrize("dense", [1.0, 0.01])
 def test_storm_cta_preaggregation(fpx, mode, dense):
     """Storms long enough for warps to warm up the CTA pre-aggregation table
-    (> 8 hit tiles per warp: 1.2e6 records on 2960 warps) and dense tiles
+    (> 8 hit tiles per warp: 1.6e6 records on 2960 warps; the dynamic tail
+    publishes the density that picks the storm kernel) and dense tiles
     (>= 4 records with events): the table equals the oracle's, so the
     shared-memory counts, the first-sighting inserts and the end-of-CTA flush
     add up exactly; and equals the per-lane ablation."""
-    p = fpxgen.Params(seed=88, n_records=1_200_001, n_sites=200, recipe=fpxgen.RECIPE_STRESS, dense_nan=dense)
+    p = fpxgen.Params(seed=88, n_records=1_600_001, n_sites=200, recipe=fpxgen.RECIPE_STRESS, dense_nan=dense)
     hdr, arena = fpxgen.generate_host(p)
     base = 7 * 10**9
     exp = oracle_scan(hdr, arena, base, mode).entries()
-    got, st, _ = gpu_scan(fpx, hdr, arena, base=base, mode=mode)
-    assert st == fpx.OK
-    assert_same(got, exp)
-    got2, _, _ = gpu_scan(fpx, hdr, arena, base=base, mode=mode, flags=fpx.OPT_NO_WARP_AGG)
-    assert_same(got2, exp)
+    for flags in (0, fpx.OPT_STORM, fpx.OPT_NO_WARP_AGG):
+        got, st, _ = gpu_scan(fpx, hdr, arena, base=base, mode=mode, flags=flags)
+        assert st == fpx.OK
+        assert_same(got, exp)
+    # adaptive kernel choice: the handle's first scan uses the sparse kernel,
+    # the density it reports switches the next ones to the storm kernel; and
+    # a sparse trace scanned after the storm is still exact
+    d_hdr, d_arena = to_dev(hdr, arena)
+    q = fpxgen.Params(seed=89, n_records=1_600_013, n_sites=500, recipe=fpxgen.RECIPE_MIX, p_fp64=0.5)
+    qh, qa = fpxgen.generate_host(q)
+    _, w = fpxgen.plan_injections(q, 500)
+    fpxgen.apply_host(w, qh, qa)
+    q_exp = oracle_scan(qh, qa, 5, DEST).entries()
+    dq_hdr, dq_arena = to_dev(qh, qa)
+    with fpx.Handle(0) as h:
+        for rep in range(3):
+            h.scan_records(d_hdr, d_arena, base_index=base, mode=mode, arena_planes=arena.shape[0])
+            assert_same(h.fetch(), exp)
+            h.reset()
+        for rep in range(2):
+            h.scan_records(dq_hdr, dq_arena, base_index=5, arena_planes=qa.shape[0])
+            assert_same(h.fetch(), q_exp)
+            h.reset()
