@@ -311,6 +311,17 @@ constexpr int kConsumeUnroll = FPX_CONSUME_UNROLL;
 #ifndef FPX_CTA_FLOW
 #define FPX_CTA_FLOW 0
 #endif
+// The sparse DEST kernel's exact path: 0 inlined, 1 a direct call, 2 through
+// g_exact_fn.  On large traces (the 20-warp ring) a call keeps the exact
+// path's code out of the scan loop's register allocation: C2 -3.1 %, C5
+// -2.6 % warp instructions, C5 +3 % throughput under the power cap; on small,
+// latency-bound traces (the 24-warp ring, C1) the inlined path is 20 % faster
+// (profiles/r2/ab_sparse_dest_call.txt).  The storm kernel always inlines.
+#ifndef FPX_SPARSE_DEST_CALL
+#define FPX_SPARSE_DEST_CALL 1
+#endif
+template <class C>
+constexpr int kSparseDestCall = C::WARPS == 24 ? 0 : FPX_SPARSE_DEST_CALL;
 // The storm machinery (CTA pre-aggregation table, storm mode) lives in a
 // separate DEST kernel instantiation (STORM = true) that the launcher picks
 // when the handle's previous launch found a storm (ScanFeedback): it costs
@@ -746,11 +757,17 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 #ifdef FPX_WARP_TIMES
       const uint64_t te0 = globaltimer_ns();
 #endif
-      if (MODE == FPX_MODE_DEST) {
+      if (MODE == FPX_MODE_DEST && (STORM || kSparseDestCall<C> == 0)) {
         const bool dense = exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes,
                                                  lane_base, sm.planes[s] + lane, lane, m.gidx0, tv, warm);
         if (kCtaTable<MODE, STORM> && lane == 0) sm.meta[0].pad[1] = dense ? min(storm_run + 1u, kStormTiles) : 0u;
-      } else if (!(tv.flags & FPX_OPT_NO_WARP_AGG))
+      } else if (MODE == FPX_MODE_DEST && kSparseDestCall<C> == 1)
+        exact_tile_ring_call<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base,
+                                   sm.planes[s] + lane, lane, m.gidx0, tv, warm);
+      else if (MODE == FPX_MODE_DEST)
+        g_exact_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
+                         lane, m.gidx0, tv, warm);
+      else if (!(tv.flags & FPX_OPT_NO_WARP_AGG))
         g_flow_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
                         lane, m.gidx0, tv, warm);
       else  // the no-aggregation ablation's record-by-record path
