@@ -138,8 +138,8 @@ constexpr uint32_t META_RESERVED = 0xFFFF80E0u;
 // shared memory of the ring kernel: per-warp rings, the decode table, the
 // CTA pre-aggregation table (fpx_device.cuh CtaTable)
 template <class C>
-constexpr size_t ring_smem() {
-  return sizeof(WarpSmem<C>) * C::WARPS + DECODE_ENTRIES + CtaTable::bytes();
+constexpr size_t ring_smem(bool cta_table = true) {
+  return sizeof(WarpSmem<C>) * C::WARPS + DECODE_ENTRIES + (cta_table ? CtaTable::bytes() : 0u);
 }
 
 // Header decode for the fast path, branch-free: validity (the contract of
@@ -810,7 +810,7 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
   if (e != cudaSuccess) return e;
   auto set_attr = [] {
     return cudaFuncSetAttribute(k_scan_records_tma<MODE, C, STORM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)ring_smem<C>());
+                                (int)ring_smem<C>(kCtaTable<MODE, STORM>));
   };
   if (dev < kMaxDevices) {
     std::call_once(once[dev], [&] { once_err[dev] = set_attr(); });
@@ -844,7 +844,7 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
     blocks = ((n + per - 1) / per + C::WARPS - 1) / C::WARPS;
   }
   if (per >= (1ull << 31)) return cudaErrorInvalidValue;  // the kernel counts a warp's records in 32 bits
-  k_scan_records_tma<MODE, C, STORM><<<(unsigned)blocks, C::WARPS * 32, ring_smem<C>(), s>>>(hdr, n, arena, arena_planes,
+  k_scan_records_tma<MODE, C, STORM><<<(unsigned)blocks, C::WARPS * 32, ring_smem<C>(kCtaTable<MODE, STORM>), s>>>(hdr, n, arena, arena_planes,
                                                                                       base_index, per, sch, tv);
   return cudaGetLastError();
 }
