@@ -312,13 +312,13 @@ constexpr int kConsumeUnroll = FPX_CONSUME_UNROLL;
 #define FPX_CTA_FLOW 0
 #endif
 // The sparse DEST kernel's exact path: 0 inlined, 1 a direct call, 2 through
-// g_exact_fn.  On large traces (the 20-warp ring) a call keeps the exact
-// path's code out of the scan loop's register allocation: C2 -3.1 %, C5
-// -2.6 % warp instructions, C5 +3 % throughput under the power cap; on small,
-// latency-bound traces (the 24-warp ring, C1) the inlined path is 20 % faster
-// (profiles/r2/ab_sparse_dest_call.txt).  The storm kernel always inlines.
+// g_exact_fn.  A call keeps the exact path's code out of the scan loop's
+// register allocation (C2 -3.1 %, C5 -2.6 % warp instructions) but the scan
+// runs 3 % slower on C2 (more stalls per instruction; interleaved bisection
+// over this round's commits, profiles/r2/bisect_c2.txt), and C1 20 % slower:
+// inlined.
 #ifndef FPX_SPARSE_DEST_CALL
-#define FPX_SPARSE_DEST_CALL 1
+#define FPX_SPARSE_DEST_CALL 0
 #endif
 template <class C>
 constexpr int kSparseDestCall = C::WARPS == 24 ? 0 : FPX_SPARSE_DEST_CALL;
