@@ -465,8 +465,15 @@ template <int MODE>
 __device__ ExactFn g_flow_fn = exact_tile_flow_call<MODE>;
 // storm mode (witnesses skipped) after this many dense exact tiles in a row
 constexpr uint32_t kStormTiles = 16;
-// the CTA table is used by a warp from its kWarmTiles-th hit tile on
-constexpr uint32_t kWarmTiles = 8;
+// the CTA table is used by a warp from its kWarmTiles-th hit tile on.  The
+// storm kernel only runs after a launch that found a storm, so it needs no
+// warm-up: 0 (8, the threshold from when one kernel served both: S1 -18 %,
+// S2 -12 %; 0 without the reconvergence below: S2 -33 %;
+// profiles/r2/ab_storm_warm.txt)
+#ifndef FPX_WARM_TILES
+#define FPX_WARM_TILES 0
+#endif
+constexpr uint32_t kWarmTiles = FPX_WARM_TILES;
 
 template <int MODE, class C, bool STORM>
 __global__ void __launch_bounds__(C::WARPS * 32, 1)
@@ -779,6 +786,11 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
         g_warp_exact_ns[gw] += globaltimer_ns() - te0;
       }
 #endif
+      // storm kernel: reconverge after the exact path.  Lanes leave it at
+      // different points (the table updates of a dense tile), and unless the
+      // warp syncs here ptxas may let the groups run the next tiles apart:
+      // S1 +3 %, S2 +4 %, and with it the warm-up can go (kWarmTiles)
+      if (STORM) __syncwarp();
     }
   }
   // out of the loop: the call's register conventions stay off the scan loop

@@ -70,7 +70,7 @@ def _oracle(n, flow, mode, base):
     return exp[mode]
 
 
-VARIANTS = [(0, "tma"), (1, "ldg"), (2, "tma-noagg"), (3, "ldg-noagg"), (8, "tma-storm")]
+VARIANTS = [(0, "tma"), (1, "ldg"), (2, "tma-noagg"), (3, "ldg-noagg"), (8, "tma-storm"), (10, "tma-storm-noagg")]
 
 
 @pytest.mark.parametrize("n", [50_011, 1_600_037], ids=["static", "dynamic"])

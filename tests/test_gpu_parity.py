@@ -146,7 +146,8 @@ def test_synthetic_trace_parity(fpx, name, recipe, mode, n, sites, variant):
         assert table_dict(got) == expected_from_injections(hdr, inj, base, mode)
 
 
-@pytest.mark.parametrize("variant", [0, 1, 2, 3], ids=["tma", "ldg", "tma-noagg", "ldg-noagg"])
+@pytest.mark.parametrize("variant", [0, 1, 2, 3, 8, 10],
+                         ids=["tma", "ldg", "tma-noagg", "ldg-noagg", "tma-storm", "tma-storm-noagg"])
 def test_dense_nan_storm(fpx, variant):
     p = fpxgen.Params(seed=77, n_records=60_000, n_sites=200, recipe=fpxgen.RECIPE_STRESS, dense_nan=1.0)
     hdr, arena = fpxgen.generate_host(p)

@@ -3,10 +3,11 @@
 capture (`ncu --set full --import-source on`): joins ncu's per-SASS-instruction
 counts with `nvdisasm -gi` line info of the same library build.
 
-    python tools/line_profile.py report.ncu-rep lib.so [kernel-substring] [--top N] [--outer]
+    python tools/line_profile.py report.ncu-rep lib.so [kernel-substring] [--top N] [--outer] [--col NAME]
 
 --outer aggregates by the outermost source line (the kernel body line an
-inlined call sits on) instead of the innermost one."""
+inlined call sits on) instead of the innermost one; --col aggregates another per-instruction column
+of the source page (e.g. "Warp Stall Sampling (All Samples)", "stall_long_sb")."""
 import collections
 import csv
 import io
@@ -20,13 +21,14 @@ rep, lib = sys.argv[1], sys.argv[2]
 ksub = sys.argv[3] if len(sys.argv) > 3 and not sys.argv[3].startswith("--") else ""
 top = int(sys.argv[sys.argv.index("--top") + 1]) if "--top" in sys.argv else 40
 outer = "--outer" in sys.argv
+col = sys.argv[sys.argv.index("--col") + 1] if "--col" in sys.argv else "Instructions Executed"
 
 txt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(txt)))
 kname = rows[0][1] if rows and len(rows[0]) > 1 else ""
 hdr = rows[1]
-ie, src = hdr.index("Instructions Executed"), hdr.index("Source")
+ie, src = hdr.index(col), hdr.index("Source")
 counts = []
 for r in rows[2:]:
     try:
@@ -75,6 +77,6 @@ tot = sum(n for n, _ in counts)
 for (n, s), (op, li, lo) in zip(counts, best):
     key = lo if outer else li
     agg[key] += n
-print(f"kernel {kname[:100]}  total warp instructions {tot}")
+print(f"kernel {kname[:100]}  total {col} {tot}")
 for k, n in agg.most_common(top):
     print(f"  {n:12d} {100 * n / tot:5.1f}%  {k}")
