@@ -386,6 +386,9 @@ __device__ __forceinline__ void consume_list(Witness& w, uint32_t b, uint32_t e,
 // counter pairs).  nchunks = 0: static ranges only.
 constexpr uint64_t kDynMinTiles = 16;  // dynamic tail only from 16 tiles per warp up
 constexpr uint32_t kDynChunk = 256;     // records per claimed chunk (8 tiles)
+// FLOW / FLOW_DETAIL: 128 (their tiles hold ~12 records with the sources, so
+// a 256-record chunk is ~21 tiles): C3 +0.9 % (profiles/r2/ab_flow_sched.txt)
+constexpr uint32_t kDynChunkFlow = 128;
 constexpr int kStaticPct = 75;          // share of the trace in static ranges (DEST)
 // FLOW / FLOW_DETAIL: a smaller static share.  Some SMs stream 1.4-1.6x
 // slower than the median (tools/warp_times.py: their warps finish 255 tiles
@@ -470,6 +473,9 @@ constexpr uint32_t kStormTiles = 16;
 // warm-up: 0 (8, the threshold from when one kernel served both: S1 -18 %,
 // S2 -12 %; 0 without the reconvergence below: S2 -33 %;
 // profiles/r2/ab_storm_warm.txt)
+#ifndef FPX_STORM_START
+#define FPX_STORM_START 1
+#endif
 #ifndef FPX_WARM_TILES
 #define FPX_WARM_TILES 0
 #endif
@@ -527,7 +533,10 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     for (int s = 0; s < STAGES; ++s) mbar_init(&sm.bar[s], 1);
     mbar_init_fence();
     sm.meta[0].pad[0] = 0u;  // hit tiles of this warp (exact path, CTA-table warm-up)
-    sm.meta[0].pad[1] = 0u;  // dense exact tiles in a row (storm mode)
+    // dense exact tiles in a row (storm mode).  The storm kernel starts in
+    // storm mode (it runs after a launch that found a storm; the first tile
+    // that is not dense turns it off)
+    sm.meta[0].pad[1] = kCtaTable<MODE, STORM> && FPX_STORM_START ? kStormTiles : 0u;
   }
   __syncwarp();
 
@@ -1009,7 +1018,7 @@ struct Tuning {
   int ring = -1;  // -1: by trace size
   int sched = 1;
   int static_pct = -1;  // -1: by mode (kStaticPct / kStaticPctFlow)
-  uint32_t dyn_chunk = kDynChunk, tail_tiles = kTailTiles;
+  uint32_t dyn_chunk = 0, tail_tiles = kTailTiles;  // dyn_chunk 0: by mode
 };
 #ifdef FPX_TUNING
 Tuning read_tuning() {
@@ -1059,7 +1068,8 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   if (ring < 0) ring = n <= (uint64_t)num_sms * 24 * TILE ? 3 : 1;
   if (tu.sched == 0) sched_ctr = nullptr;
   const int static_pct = tu.static_pct >= 0 ? tu.static_pct : MODE == FPX_MODE_DEST ? kStaticPct : kStaticPctFlow;
-  const SchedCfg scfg{static_pct, tu.dyn_chunk, tu.sched == 2 ? 0u : tu.tail_tiles};
+  const uint32_t chunk = tu.dyn_chunk ? tu.dyn_chunk : MODE == FPX_MODE_DEST ? kDynChunk : kDynChunkFlow;
+  const SchedCfg scfg{static_pct, chunk, tu.sched == 2 ? 0u : tu.tail_tiles};
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   if constexpr (MODE == FPX_MODE_DEST) {
     if (storm) {  // the storm instantiation (CTA table, storm mode)
