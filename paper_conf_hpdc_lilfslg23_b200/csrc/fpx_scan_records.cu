@@ -317,6 +317,15 @@ constexpr int kConsumeUnroll = FPX_CONSUME_UNROLL;
 // runs 3 % slower on C2 (more stalls per instruction; interleaved bisection
 // over this round's commits, profiles/r2/bisect_c2.txt), and C1 20 % slower:
 // inlined.
+// The analyzer kernels' exact path: 1 = the lean path (exact_tile_flow)
+// inlined, 0 = called through g_flow_fn, 2 = the generic record path inlined.
+// Inlined, ptxas spills 40 B on the rare exact path, but the call (an ABI
+// frame in the scan loop) cost C3 0.8 % with the FLOW work split and 4.5 %
+// with the DEST one (profiles/r2/ab_flow_inline.txt; bisected to the commit
+// that introduced the call, profiles/r2/bisect_c3.txt).
+#ifndef FPX_FLOW_INLINE
+#define FPX_FLOW_INLINE 1
+#endif
 #ifndef FPX_SPARSE_DEST_CALL
 #define FPX_SPARSE_DEST_CALL 0
 #endif
@@ -783,9 +792,22 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       else if (MODE == FPX_MODE_DEST)
         g_exact_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
                          lane, m.gidx0, tv, warm);
-      else if (!(tv.flags & FPX_OPT_NO_WARP_AGG))
+      else if (!(tv.flags & FPX_OPT_NO_WARP_AGG)) {
+#if FPX_FLOW_INLINE == 2
+        exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base,
+                              sm.planes[s] + lane, lane, m.gidx0, tv, warm);
+#elif FPX_FLOW_INLINE
+        exact_tile_flow<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base,
+                              sm.planes[s] + lane, lane, m.gidx0, tv, warm, [](uint32_t meta) {
+                                bool f;
+                                const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, f, f);
+                                return fmt_of(meta) == FPX_FP64 ? 2u * ni : ni;
+                              });
+#else
         g_flow_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
                         lane, m.gidx0, tv, warm);
+#endif
+      }
       else  // the no-aggregation ablation's record-by-record path
         g_exact_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
                          lane, m.gidx0, tv, warm);
