@@ -57,6 +57,11 @@ constexpr uint32_t TV_SHARED = 1u << 16;
 // (ctl->live; FPX_OPT_LIVE_NEW on the home handle; never on attached ones,
 // whose process cannot see the home's host ring).
 constexpr uint32_t TV_LIVE = 1u << 17;
+// TableView::flags bit, set per launch by the sparse record-scan kernels'
+// launcher: table_add tries the key's home slot with the CAS straight away
+// (most of their events are new keys); storm kernels, whose events mostly hit
+// present hot keys, and the per-lane ablation read the slot first.
+constexpr uint32_t TV_CAS_FIRST = 1u << 18;
 
 // Everything a scan kernel needs to update the table, passed by value.
 struct TableView {
@@ -66,7 +71,7 @@ struct TableView {
   unsigned int* newlog_slot;     // slot index of each logged key (for the touched-slot reset)
   unsigned long long newlog_cap;
   Ctl* ctl;
-  uint32_t flags;                // FPX_OPT_NO_WARP_AGG (ablation) | TV_SHARED | TV_LIVE
+  uint32_t flags;                // FPX_OPT_NO_WARP_AGG (ablation) | TV_SHARED | TV_LIVE | TV_CAS_FIRST
 };
 
 // One tensor of a fused multi-tensor scan (host-prepared, device-resident).

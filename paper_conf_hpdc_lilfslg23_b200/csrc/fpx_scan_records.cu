@@ -326,6 +326,9 @@ constexpr int kConsumeUnroll = FPX_CONSUME_UNROLL;
 #ifndef FPX_FLOW_INLINE
 #define FPX_FLOW_INLINE 1
 #endif
+#ifndef FPX_CAS_FIRST
+#define FPX_CAS_FIRST 1  // TV_CAS_FIRST for the sparse kernels (fpx_internal.h)
+#endif
 #ifndef FPX_SPARSE_DEST_CALL
 #define FPX_SPARSE_DEST_CALL 0
 #endif
@@ -1103,11 +1106,14 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
       }
     }
   }
+  // sparse kernels: new keys dominate their table updates (TV_CAS_FIRST)
+  TableView tvs = tv;
+  if (FPX_CAS_FIRST && !(tv.flags & FPX_OPT_NO_WARP_AGG)) tvs.flags |= TV_CAS_FIRST;
   switch (ring) {
-    case 1: return launch_ring<MODE, Ring1, false>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
-    case 2: return launch_ring<MODE, Ring2, false>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
-    case 3: return launch_ring<MODE, Ring3, false>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
-    default: return launch_ring<MODE, Ring0, false>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
+    case 1: return launch_ring<MODE, Ring1, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
+    case 2: return launch_ring<MODE, Ring2, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
+    case 3: return launch_ring<MODE, Ring3, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
+    default: return launch_ring<MODE, Ring0, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
   }
 }
 
