@@ -109,8 +109,12 @@ constexpr int NLISTS = 8;
 
 // StageMeta::k bit 31: the tile holds a record that must take the exact path
 constexpr uint32_t kForceBit = 0x80000000u;
+// StageMeta::k bit 30: the producer built no item lists (a storm kernel warp
+// in storm mode): the tile goes to the exact path
+constexpr uint32_t kNoListBit = 0x40000000u;
+constexpr uint32_t kFlagBits = kForceBit | kNoListBit;
 struct StageMeta {
-  uint32_t k;      // records in the tile (0 = no tile) | kForceBit
+  uint32_t k;      // records in the tile (0 = no tile) | kForceBit | kNoListBit
   uint32_t tot;    // items in the tile (end of the last list)
   uint64_t gidx0;  // global index of the tile's first record
   uint32_t sb;     // byte f: first item of format f's full-mask list
@@ -485,6 +489,9 @@ constexpr uint32_t kStormTiles = 16;
 // warm-up: 0 (8, the threshold from when one kernel served both: S1 -18 %,
 // S2 -12 %; 0 without the reconvergence below: S2 -33 %;
 // profiles/r2/ab_storm_warm.txt)
+#ifndef FPX_STORM_NO_LISTS
+#define FPX_STORM_NO_LISTS 1
+#endif
 #ifndef FPX_STORM_START
 #define FPX_STORM_START 1
 #endif
@@ -633,7 +640,9 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     // f's full-mask list).  Every byte stays <= 40 (items <= planes), so the
     // packed sums never carry.
     const uint32_t below = (tot_f * 0x01010101u) << 8;
-    const bool writes = in_tile && ni != 0u;
+    // storm mode: the consumer skips the witnesses, so the lists are not built
+    const bool lists = !kCtaTable<MODE, STORM> || !FPX_STORM_NO_LISTS || sm.meta[0].pad[1] < kStormTiles;
+    const bool writes = lists && in_tile && ni != 0u;
     uint32_t at = 0u;
     if (writes) {
       // byte f of `own`: this record's place among format f's items (full list first)
@@ -653,7 +662,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
         if (writes && j < ni) sm.items[s][at + j] = make_uint2(slot + j * step, mask);
     }
     if (lane == 0) {
-      m.k = k | (force_any != 0u ? kForceBit : 0u);
+      m.k = k | (force_any != 0u ? kForceBit : 0u) | (lists ? 0u : kNoListBit);
       m.gidx0 = base_index + cursor;
       m.sb = below;              // list starts, packed (consumer: one PRMT per bound)
       m.sp = below + tf;
@@ -709,7 +718,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const int s = (int)(i % STAGES);
     produce((int)((i + STAGES - 1) % STAGES));
     const StageMeta& m = sm.meta[s];
-    const uint32_t mk = m.k;  // records in the tile | kForceBit
+    const uint32_t mk = m.k;  // records in the tile | kForceBit | kNoListBit
     if (mk == 0u) {
 #ifdef FPX_WARP_TIMES
       if (lane == 0 && gw < kMaxWarpTimes) g_warp_t1[gw] = globaltimer_ns();
@@ -751,7 +760,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     // (the run length lives in the stage-0 descriptor's spare word: a register
     // held across the loop cost S2 6 %, profiles/r2/ab_storm_state.txt)
     const uint32_t storm_run = kCtaTable<MODE, STORM> ? sm.meta[0].pad[1] : 0u;
-    bool hit = kCtaTable<MODE, STORM> && storm_run >= kStormTiles;
+    bool hit = kCtaTable<MODE, STORM> && (storm_run >= kStormTiles || (mk & kNoListBit) != 0u);
     if (!hit) {
       // ---- fast path over the staged planes (lane-quad layout) ------------
       const uint32_t ia = smem_u32(sm.items[s]), pa = smem_u32(sm.planes[s]);
@@ -786,33 +795,33 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       const uint64_t te0 = globaltimer_ns();
 #endif
       if (MODE == FPX_MODE_DEST && (STORM || kSparseDestCall<C> == 0)) {
-        const bool dense = exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes,
+        const bool dense = exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes,
                                                  lane_base, sm.planes[s] + lane, lane, m.gidx0, tv, warm);
         if (kCtaTable<MODE, STORM> && lane == 0) sm.meta[0].pad[1] = dense ? min(storm_run + 1u, kStormTiles) : 0u;
       } else if (MODE == FPX_MODE_DEST && kSparseDestCall<C> == 1)
-        exact_tile_ring_call<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base,
+        exact_tile_ring_call<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes, lane_base,
                                    sm.planes[s] + lane, lane, m.gidx0, tv, warm);
       else if (MODE == FPX_MODE_DEST)
-        g_exact_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
+        g_exact_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes, lane_base, sm.planes[s] + lane,
                          lane, m.gidx0, tv, warm);
       else if (!(tv.flags & FPX_OPT_NO_WARP_AGG)) {
 #if FPX_FLOW_INLINE == 2
-        exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base,
+        exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes, lane_base,
                               sm.planes[s] + lane, lane, m.gidx0, tv, warm);
 #elif FPX_FLOW_INLINE
-        exact_tile_flow<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base,
+        exact_tile_flow<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes, lane_base,
                               sm.planes[s] + lane, lane, m.gidx0, tv, warm, [](uint32_t meta) {
                                 bool f;
                                 const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, f, f);
                                 return fmt_of(meta) == FPX_FP64 ? 2u * ni : ni;
                               });
 #else
-        g_flow_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
+        g_flow_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes, lane_base, sm.planes[s] + lane,
                         lane, m.gidx0, tv, warm);
 #endif
       }
       else  // the no-aggregation ablation's record-by-record path
-        g_exact_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kForceBit, arena_planes, lane_base, sm.planes[s] + lane,
+        g_exact_fn<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes, lane_base, sm.planes[s] + lane,
                          lane, m.gidx0, tv, warm);
 #ifdef FPX_WARP_TIMES
       if (lane == 0 && gw < kMaxWarpTimes) {
