@@ -489,6 +489,9 @@ constexpr uint32_t kStormTiles = 16;
 // warm-up: 0 (8, the threshold from when one kernel served both: S1 -18 %,
 // S2 -12 %; 0 without the reconvergence below: S2 -33 %;
 // profiles/r2/ab_storm_warm.txt)
+#ifndef FPX_POLICY_PER_TILE
+#define FPX_POLICY_PER_TILE 0  // 1: recomputed per tile (no spill in the sparse DEST kernel, but C2 / C5 -0.5-1.2 %: ab_policy.txt)
+#endif
 #ifndef FPX_STORM_NO_LISTS
 #define FPX_STORM_NO_LISTS 1
 #endif
@@ -544,7 +547,9 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   if (sch.nchunks != 0u && lane == 0) claim = atomicAdd(sch.ctr, 1u);
   const uint32_t* __restrict__ lane_base = arena + lane;
   const uint4* __restrict__ hdr_lane = hdr + lane;  // this lane's header of a tile = hdr_lane[tile start]
+#if !FPX_POLICY_PER_TILE
   const uint64_t policy = policy_evict_first();
+#endif
   const uint32_t g = (uint32_t)lane >> 3, q = (uint32_t)lane & 7u;
 
   if (lane == 0) {
@@ -682,6 +687,9 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     if (one_run) {
       if (lane == 0) {
         mbar_arrive_expect_tx(&sm.bar[s], total * 128u);
+#if FPX_POLICY_PER_TILE
+        const uint64_t policy = policy_evict_first();  // one instruction; not a register held by the scan loop
+#endif
         if (total != 0u) bulk_g2s(&sm.planes[s][0], arena + (uint64_t)dmin * 32, total * 128u, &sm.bar[s], policy);
       }
     } else {
@@ -701,7 +709,12 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       if (lane == 0) mbar_arrive_expect_tx(&sm.bar[s], total * 128u);
       __syncwarp();
       if (head)
+      {
+#if FPX_POLICY_PER_TILE
+        const uint64_t policy = policy_evict_first();
+#endif
         bulk_g2s(&sm.planes[s][slot * 32], arena + (uint64_t)a * 32, (run_end - slot) * 128u, &sm.bar[s], policy);
+      }
     }
     // advance and prefetch the next tile's headers
     cursor += k;
