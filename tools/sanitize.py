@@ -1,6 +1,7 @@
 """Small scans of every kernel family for compute-sanitizer (memcheck,
 racecheck, synccheck): DEST / FLOW / FLOW_DETAIL record scans (TMA ring and
-LDG), the record scan's dynamic tail, a storm trace (exact path + table atomics), tensor scans with ragged
+LDG), the record scan's dynamic tail, storm traces through the sparse and the
+storm DEST kernels (exact path, CTA table, table atomics), tensor scans with ragged
 heads / tails, fetch / FETCH_NEW / reset / merge paths."""
 import os
 import sys
@@ -41,17 +42,23 @@ with fpx.Handle(0) as h:
 del hdr, arena
 p = fpxgen.Params(seed=9, n_records=5000, n_sites=20, recipe=fpxgen.RECIPE_STRESS, dense_nan=1.0)
 hdr, arena, planes = fpxgen.generate_device(p)
-with fpx.Handle(0, table_log2_slots=5) as h:
-    h.scan_records(hdr, arena, arena_planes=planes)
-    h.fetch()
-# storms long enough for warm warps: the CTA pre-aggregation table (shared
-# atomics from 20 warps, end-of-CTA flush by the last warp), DEST and FLOW
-p = fpxgen.Params(seed=10, n_records=900_017, n_sites=40, recipe=fpxgen.RECIPE_STRESS, dense_nan=0.05)
-hdr, arena, planes = fpxgen.generate_device(p)
-for mode in (0, 1):
-    with fpx.Handle(0) as h:
-        h.scan_records(hdr, arena, mode=mode, arena_planes=planes)
+for flags in (0, fpx.OPT_STORM):  # the small-trace ring: sparse and storm DEST kernels
+    with fpx.Handle(0, table_log2_slots=5, flags=flags) as h:
+        h.scan_records(hdr, arena, arena_planes=planes)
         h.fetch()
+# storms: the storm DEST kernel (CTA pre-aggregation table: shared atomics from
+# 20 warps, end-of-CTA flush by the last warp; storm mode without item lists),
+# picked by the density feedback of the first launch on the handle (and
+# forced); FLOW; the dynamic tail of the storm kernel (1.6 M records)
+for n, dense in ((900_017, 0.05), (1_600_037, 0.02)):
+    p = fpxgen.Params(seed=10, n_records=n, n_sites=40, recipe=fpxgen.RECIPE_STRESS, dense_nan=dense)
+    hdr, arena, planes = fpxgen.generate_device(p)
+    for mode, flags in ((0, 0), (0, fpx.OPT_STORM), (1, 0)):
+        with fpx.Handle(0, flags=flags) as h:
+            for _ in range(2):
+                h.scan_records(hdr, arena, mode=mode, arena_planes=planes)
+                torch.cuda.synchronize()  # the second launch reads the first one's feedback
+            h.fetch()
 # early notification ring (mapped host memory) and a shared (exported) table
 with fpx.Handle(0, flags=fpx.OPT_LIVE_NEW) as h:
     h.export()
