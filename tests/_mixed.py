@@ -72,11 +72,13 @@ def _masks(rng, n):
     return np.where(u < 0.45, full, np.where(u < 0.8, partial, np.where(u < 0.95, sparse, 0))).astype(np.uint32)
 
 
-def zoo_trace(seed: int, n: int, flow: bool, n_sites: int = 13, p_bad_flow: float = 0.02):
+def zoo_trace(seed: int, n: int, flow: bool, n_sites: int = 13, p_bad_flow: float = 0.02,
+              levels=((0.0, 0.02, 0.25, 0.9), (0.55, 0.2, 0.15, 0.1))):
     """(hdr, arena) of n zoo records.  flow=True shapes records for the
     analyzer (scalar FP32 / FP64, destination width 0 or one value) except a
     share p_bad_flow of packed records, which the FLOW modes must count as bad
-    (reading R13); flow=False draws every legal DEST record shape."""
+    (reading R13); flow=False draws every legal DEST record shape.  `levels`:
+    the per-block special-value shares and their probabilities."""
     rng = np.random.default_rng(seed)
     op = rng.integers(0, 20, size=n)
     if flow:
@@ -100,7 +102,7 @@ def zoo_trace(seed: int, n: int, flow: bool, n_sites: int = 13, p_bad_flow: floa
     # per block of 40 records: how exceptional the values are (clean stretches
     # keep whole tiles on the fast path; dense stretches mix many codes)
     blocks = (n + 39) // 40
-    p_blk = rng.choice([0.0, 0.02, 0.25, 0.9], size=blocks, p=[0.55, 0.2, 0.15, 0.1])
+    p_blk = rng.choice(list(levels[0]), size=blocks, p=list(levels[1]))
     p_rec = p_blk[np.arange(n) // 40]
     mask = _masks(rng, n)
     hdr = np.zeros(n, dtype=HDR_DTYPE)
@@ -197,3 +199,12 @@ def isolated_fp64_trace(values: np.ndarray, opclass: int = 9, filler: int = 0x3F
     arena[2 * carriers, lane] = (v & np.uint64(0xFFFFFFFF)).astype(np.uint32)
     arena[2 * carriers + 1, lane] = (v >> np.uint64(32)).astype(np.uint32)
     return hdr, arena
+
+
+def sparse_flow_trace(seed: int, n: int):
+    """Analyzer-shaped zoo records whose special values are rare (a share
+    0.002 in half of the 40-record blocks): a hit tile then holds one or two
+    records with an exceptional destination or source -- in any plane, FP32
+    or either word of an FP64 pair, active or not -- among clean ones, the
+    case the analyzer's candidate filter (exact_tile_flow) skips records in."""
+    return zoo_trace(seed, n, flow=True, levels=((0.0, 0.002), (0.5, 0.5)))

@@ -14,7 +14,7 @@ import numpy as np
 import pytest
 
 import oracle
-from _mixed import isolated_fp64_trace, isolated_word_trace, zoo_trace
+from _mixed import isolated_fp64_trace, isolated_word_trace, sparse_flow_trace, zoo_trace
 from _records import (
     BF16, DEST, FLOW, FLOW_DETAIL, FP16, FP32, FP64, NONE, describe_diff, entries_equal, np_class, table_dict,
 )
@@ -91,6 +91,26 @@ def test_zoo_parity(fpx, n, mode, flags):
     assert flows == ({NONE} if mode == DEST else {1, 2, 3})
     if mode == FLOW_DETAIL:
         assert {int(e["detail"]) for e in exp} >= {0, 1, 2, 3, 5, 6, 7}
+
+
+@pytest.mark.parametrize("n", [200_003, 1_600_037], ids=["static", "dynamic"])
+@pytest.mark.parametrize("mode", [FLOW, FLOW_DETAIL], ids=["flow", "flow_detail"])
+@pytest.mark.parametrize("flags", [0, 1], ids=["tma", "ldg"])
+def test_flow_sparse_candidates(fpx, n, mode, flags):
+    """Hit analyzer tiles with one or two exceptional records among clean
+    ones: the exact path walks only the records with a candidate plane
+    (flow_candidates); the table must still equal the oracle's."""
+    hdr, arena = sparse_flow_trace(seed=77 + n, n=n)
+    base = 12345
+    t = oracle.Table()
+    t.scan_records(hdr, arena, base_index=base, mode=mode)
+    exp = t.entries()
+    got, stats = gpu_table(fpx, hdr, arena, base, mode, flags)
+    assert entries_equal(got, exp), describe_diff(got, exp)
+    assert stats.bad_records == t.bad_records
+    assert {int(e["flow"]) for e in exp} == {1, 2, 3}
+    # sparse: far fewer events than records
+    assert int(np.sum(exp["count"])) < n // 4
 
 
 # ---------------------------------------------------------------------------
