@@ -337,13 +337,125 @@ static __device__ __noinline__ void cta_warp_done(const TableView tv, uint32_t n
   }
 }
 
+// Per-CTA table-update queue (the analyzer kernels): the scan warps hand
+// their warp-reduced (key, count, first) events to one extra warp of the CTA,
+// the drain warp, which issues them (table_add) while the scan warps go on
+// streaming.  A table insert costs one or two dependent L2 round trips (the
+// key CAS, then the new-key log position), ~2 us each under a full HBM
+// stream: half of an analyzer hit tile's time when the scanning warp waited
+// for them itself (profiles/r2/ab_flow_cand.txt).  Same updates, same table;
+// only the issuing warp changes.  A bounded ring of tickets: a producer lane
+// takes ticket t from `tail` (shared atomic), waits until entry t % EQ_N is
+// free for it (seq == t; only when EQ_N events are in flight), writes the
+// event and publishes seq = t + 1; the drain warp takes tickets in order, 32
+// at a time (one lane each, so up to 32 inserts overlap), and frees each
+// entry for ticket t + EQ_N.  The image sits at the END of dynamic shared
+// memory (found from %dynamic_smem_size, like CtaTable; the kernels that use
+// the queue have no CTA table).
+constexpr uint32_t EQ_N = 256;  // entries (power of two)
+struct EqEntry {
+  unsigned long long key, first;
+  uint32_t count, seq;
+};
+static_assert(sizeof(EqEntry) == 24, "queue entry");
+struct EventQueue {
+  EqEntry* e;          // [EQ_N]
+  unsigned int* hdr;   // [0] tail (tickets taken), [1] scan warps done
+  __host__ __device__ static constexpr size_t bytes() { return EQ_N * sizeof(EqEntry) + 16; }
+  __device__ static EventQueue from_image() {
+    extern __shared__ __align__(128) uint8_t fpx_dyn_smem[];
+    uint32_t dyn;
+    asm("mov.u32 %0, %%dynamic_smem_size;" : "=r"(dyn));
+    uint8_t* p = fpx_dyn_smem + dyn - bytes();
+    return EventQueue{reinterpret_cast<EqEntry*>(p), reinterpret_cast<unsigned int*>(p + EQ_N * sizeof(EqEntry))};
+  }
+  // by the whole CTA, before a __syncthreads
+  __device__ void init() const {
+    for (uint32_t i = threadIdx.x; i < EQ_N; i += blockDim.x) e[i].seq = i;
+    if (threadIdx.x == 0) hdr[0] = hdr[1] = 0u;
+  }
+};
+
+// Bounded spin of the queue's hand-offs: the other side is always running (a
+// producer writes right after taking its ticket; the drain warp frees entries
+// as it goes), so a 4 s stall is an internal bug -- a launch error, not a hang.
+__device__ __forceinline__ void eq_stall_check(unsigned long long& t0) {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  if (t0 == 0ull) t0 = t;
+  else if (t - t0 > 4000000000ull) __trap();
+}
+
+// One event into the CTA's queue (any lane; divergent callers welcome).
+// Out of line: the scan loop's register budget stays with the fast path.
+static __device__ __noinline__ void eq_push(unsigned long long key, uint32_t c, unsigned long long f) {
+  const EventQueue q = EventQueue::from_image();
+  const uint32_t t = atomicAdd(q.hdr, 1u);
+  EqEntry* e = q.e + (t & (EQ_N - 1u));
+  unsigned long long t0 = 0ull;
+  while (*reinterpret_cast<volatile uint32_t*>(&e->seq) != t) {  // queue full: wait for the drain
+    __nanosleep(64);
+    eq_stall_check(t0);
+  }
+  e->key = key;
+  e->first = f;
+  e->count = c;
+  __threadfence_block();
+  *reinterpret_cast<volatile uint32_t*>(&e->seq) = t + 1u;
+}
+
+// A scan warp is done pushing (warp-uniform, once per scan warp, including
+// warps without work).
+static __device__ __forceinline__ void eq_warp_done() {
+  __syncwarp();
+  __threadfence_block();
+  if ((threadIdx.x & 31u) == 0u) atomicAdd(EventQueue::from_image().hdr + 1, 1u);
+}
+
+// The drain warp: issues every queued event until all `nscan` scan warps are
+// done and the queue is empty.
+static __device__ __noinline__ void eq_drain(const TableView tv, uint32_t nscan) {
+  const EventQueue q = EventQueue::from_image();
+  const uint32_t lane = threadIdx.x & 31u;
+  volatile unsigned int* vh = q.hdr;
+  uint32_t h = 0u;
+  for (;;) {
+    uint32_t t = vh[0];
+    if (t == h) {
+      if (vh[1] != nscan) {
+        __nanosleep(256);
+        continue;
+      }
+      __threadfence_block();
+      t = vh[0];  // every push of a done warp took its ticket before the warp counted itself done
+      if (t == h) break;
+    }
+    const uint32_t n = min(t - h, 32u);
+    if (lane < n) {
+      EqEntry* e = q.e + ((h + lane) & (EQ_N - 1u));
+      unsigned long long t0 = 0ull;
+      while (*reinterpret_cast<volatile uint32_t*>(&e->seq) != h + lane + 1u) eq_stall_check(t0);
+      __threadfence_block();
+      const unsigned long long key = *reinterpret_cast<volatile unsigned long long*>(&e->key);
+      const unsigned long long f = *reinterpret_cast<volatile unsigned long long*>(&e->first);
+      const uint32_t c = *reinterpret_cast<volatile uint32_t*>(&e->count);
+      __threadfence_block();
+      *reinterpret_cast<volatile uint32_t*>(&e->seq) = h + lane + EQ_N;  // free for ticket h + lane + EQ_N
+      table_add(tv, key, c, f);
+    }
+    __syncwarp();
+    h += n;
+  }
+}
+
 // Table updates of one warp, batched: the warp-reduced (key, count, first)
 // events of a tile are parked one per lane and issued by up to 32 lanes at
 // once, so a dense tile (storms) costs ~one L2 round trip per 32 events
 // instead of one per event.  Consecutive events with the same key (a storm
 // over one site) merge before any atomic.  `n` and `last` are warp-uniform.
 // CTA = true: the issued events go through emit_event (CTA table).
-template <bool CTA = false>  // CTA: issue through emit_event (ring kernel only)
+// Q = true: hand the events to the CTA's drain warp (eq_push) instead.
+template <bool CTA = false, bool Q = false>  // CTA: issue through emit_event (ring kernel only)
 struct PendingEvents {
   unsigned long long key = 0, first = 0, last = FPX_KEY_EMPTY;
   uint32_t count = 0, n = 0;
@@ -372,7 +484,8 @@ struct PendingEvents {
   __device__ __forceinline__ void flush(const TableView& tv) {
     const bool dense = warm && n >= kDenseEvents;  // warp-uniform
     if ((threadIdx.x & 31) < n) {
-      if (CTA) emit_event(tv, key, count, first, dense);
+      if (Q) eq_push(key, count, first);
+      else if (CTA) emit_event(tv, key, count, first, dense);
       else table_add(tv, key, count, first);
     }
     n = 0;

@@ -142,8 +142,10 @@ constexpr uint32_t META_RESERVED = 0xFFFF80E0u;
 // shared memory of the ring kernel: per-warp rings, the decode table, the
 // CTA pre-aggregation table (fpx_device.cuh CtaTable)
 template <class C>
-constexpr size_t ring_smem(bool cta_table = true) {
-  return sizeof(WarpSmem<C>) * C::WARPS + DECODE_ENTRIES + (cta_table ? CtaTable::bytes() : 0u);
+constexpr size_t ring_smem(bool cta_table = true, bool eq = false) {
+  // with the event queue the last warp drains it and has no ring
+  return sizeof(WarpSmem<C>) * (C::WARPS - (eq ? 1 : 0)) + DECODE_ENTRIES + (cta_table ? CtaTable::bytes() : 0u) +
+         (eq ? EventQueue::bytes() : 0u);
 }
 
 // Header decode for the fast path, branch-free: validity (the contract of
@@ -345,6 +347,19 @@ constexpr int kSparseDestCall = C::WARPS == 24 ? 0 : FPX_SPARSE_DEST_CALL;
 // on storms.  The analyzer kernels never use it (it cost 5 % of C3).
 template <int MODE, bool STORM>
 constexpr bool kCtaTable = STORM && (MODE == FPX_MODE_DEST || FPX_CTA_FLOW);
+// In the analyzer kernels the last warp of each CTA is the drain warp: it
+// issues the exact path's table updates (fpx_device.cuh EventQueue), so the
+// scan warps do not wait for the inserts' L2 round trips.  It replaces a scan
+// warp rather than adding one: a 21st warp puts 6 warps on one SM
+// sub-partition and caps the kernel at 80 registers (spills in the scan
+// loop).  0: every warp scans and issues its own updates (A/B).
+#ifndef FPX_EQ
+#define FPX_EQ 1
+#endif
+template <int MODE, bool STORM>
+constexpr bool kEq = FPX_EQ && MODE != FPX_MODE_DEST && !kCtaTable<MODE, STORM>;
+template <int MODE, class C, bool STORM>
+constexpr int kScanWarps = C::WARPS - (kEq<MODE, STORM> ? 1 : 0);
 #ifndef FPX_BAD_SYS
 #define FPX_BAD_SYS 1
 #endif
@@ -484,6 +499,17 @@ template <int MODE>
 __device__ ExactFn g_flow_fn = exact_tile_flow_call<MODE>;
 // storm mode (witnesses skipped) after this many dense exact tiles in a row
 constexpr uint32_t kStormTiles = 16;
+// Hysteresis of storm mode: a dense tile adds 1 to the run (up to kStormCap),
+// a tile that is not dense takes kStormDrop off; storm mode while the run is
+// >= kStormTiles.  On the 1 % storm S2 about one tile in 75 has fewer than 4
+// records with an event: resetting the run on it sent ~17 % of S2's tiles
+// through the fast path and its lists before the exact path (line profile,
+// profiles/r2/lines_s2_r2v5.txt).  Leaving a storm costs (kStormCap -
+// kStormTiles) / kStormDrop + 1 = 3 extra exact tiles.
+#ifndef FPX_STORM_CAP
+#define FPX_STORM_CAP 24
+#endif
+constexpr uint32_t kStormCap = FPX_STORM_CAP, kStormDrop = 4;
 // the CTA table is used by a warp from its kWarmTiles-th hit tile on.  The
 // storm kernel only runs after a launch that found a storm, so it needs no
 // warm-up: 0 (8, the threshold from when one kernel served both: S1 -18 %,
@@ -515,7 +541,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   uint8_t* rings = fpx_dyn_smem;
   WarpSmem<C>& sm = reinterpret_cast<WarpSmem<C>*>(rings)[warp];
-  uint8_t* lut = rings + sizeof(WarpSmem<C>) * C::WARPS;
+  uint8_t* lut = rings + sizeof(WarpSmem<C>) * kScanWarps<MODE, C, STORM>;
   build_decode_table<MODE>(lut);
   // CTA pre-aggregation of the exact path's table updates (fpx_device.cuh
   // CtaTable; the exact path finds it through emit_event); off for the
@@ -524,11 +550,18 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   if (kCtaTable<MODE, STORM>)
     CtaTable{reinterpret_cast<unsigned long long*>(CtaTable::image_at()), base_index}
         .init((tv.flags & FPX_OPT_NO_WARP_AGG) == 0u && n < (uint64_t)CT_NONE);
+  if (kEq<MODE, STORM>) EventQueue::from_image().init();
   __syncthreads();
-  const uint64_t gw = blockIdx.x * (uint64_t)C::WARPS + warp;
+  constexpr int SW = kScanWarps<MODE, C, STORM>;
+  if (kEq<MODE, STORM> && warp == SW) {  // the drain warp (no block-wide barriers below)
+    eq_drain(tv, SW);
+    return;
+  }
+  const uint64_t gw = blockIdx.x * (uint64_t)SW + warp;
   const uint64_t start = gw * recs_per_warp;
   if (start >= n) {  // warp-uniform; no block-wide barriers below this line
     if (kCtaTable<MODE, STORM>) cta_warp_done(tv, C::WARPS);
+    if (kEq<MODE, STORM>) eq_warp_done();
     return;
   }
 #ifdef FPX_WARP_TIMES
@@ -557,10 +590,10 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     for (int s = 0; s < STAGES; ++s) mbar_init(&sm.bar[s], 1);
     mbar_init_fence();
     sm.meta[0].pad[0] = 0u;  // hit tiles of this warp (exact path, CTA-table warm-up)
-    // dense exact tiles in a row (storm mode).  The storm kernel starts in
-    // storm mode (it runs after a launch that found a storm; the first tile
-    // that is not dense turns it off)
-    sm.meta[0].pad[1] = kCtaTable<MODE, STORM> && FPX_STORM_START ? kStormTiles : 0u;
+    // the storm run (storm mode, kStormCap).  The storm kernel starts in
+    // storm mode (it runs after a launch that found a storm; tiles that are
+    // not dense wear it off)
+    sm.meta[0].pad[1] = kCtaTable<MODE, STORM> && FPX_STORM_START ? kStormCap : 0u;
   }
   __syncwarp();
 
@@ -769,7 +802,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 
     // Storm mode (DEST): after kStormTiles dense exact tiles in a row a warp
     // skips the witnesses -- in a storm every tile is hit anyway -- and
-    // sends each tile straight to the exact path, until one is not dense.
+    // sends each tile straight to the exact path, until tiles that are not
+    // dense bring the run below kStormTiles (hysteresis: kStormCap).
     // (the run length lives in the stage-0 descriptor's spare word: a register
     // held across the loop cost S2 6 %, profiles/r2/ab_storm_state.txt)
     const uint32_t storm_run = kCtaTable<MODE, STORM> ? sm.meta[0].pad[1] : 0u;
@@ -810,7 +844,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       if (MODE == FPX_MODE_DEST && (STORM || kSparseDestCall<C> == 0)) {
         const bool dense = exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes,
                                                  lane_base, sm.planes[s] + lane, lane, m.gidx0, tv, warm);
-        if (kCtaTable<MODE, STORM> && lane == 0) sm.meta[0].pad[1] = dense ? min(storm_run + 1u, kStormTiles) : 0u;
+        if (kCtaTable<MODE, STORM> && lane == 0)
+          sm.meta[0].pad[1] = dense ? min(storm_run + 1u, kStormCap) : storm_run - min(storm_run, kStormDrop);
       } else if (MODE == FPX_MODE_DEST && kSparseDestCall<C> == 1)
         exact_tile_ring_call<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes, lane_base,
                                    sm.planes[s] + lane, lane, m.gidx0, tv, warm);
@@ -822,7 +857,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
         exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes, lane_base,
                               sm.planes[s] + lane, lane, m.gidx0, tv, warm);
 #elif FPX_FLOW_INLINE
-        exact_tile_flow<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes, lane_base,
+        exact_tile_flow<MODE, kEq<MODE, STORM>>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes, lane_base,
                               sm.planes[s] + lane, lane, m.gidx0, tv, warm, [](uint32_t meta) {
                                 bool f;
                                 const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, f, f);
@@ -851,6 +886,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   }
   // out of the loop: the call's register conventions stay off the scan loop
   if (kCtaTable<MODE, STORM>) cta_warp_done(tv, C::WARPS);
+  if (kEq<MODE, STORM>) eq_warp_done();
 }
 
 // Ring configurations compiled in; FPX_RING (environment, tuning only) picks
@@ -859,9 +895,15 @@ using Ring0 = RingCfg<16, 2, 50>;
 using Ring1 = RingCfg<20, 2, 40>;
 using Ring2 = RingCfg<28, 2, 28>;
 using Ring3 = RingCfg<24, 2, 32>;
+// the analyzer kernels with the drain warp (kEq): 19 scan warps x 42 planes
+// keep Ring1's bytes in flight
+using Ring1E = RingCfg<20, 2, 42>;
 static_assert(sizeof(WarpSmem<Ring2>) % 128 == 0 && ring_smem<Ring0>() <= 227 * 1024 && ring_smem<Ring1>() <= 227 * 1024 &&
                   ring_smem<Ring2>() <= 227 * 1024 && ring_smem<Ring3>() <= 227 * 1024,
               "ring exceeds shared memory");
+static_assert(ring_smem<Ring0>(false, true) <= 227 * 1024 && ring_smem<Ring1E>(false, true) <= 227 * 1024 &&
+                  ring_smem<Ring2>(false, true) <= 227 * 1024 && ring_smem<Ring3>(false, true) <= 227 * 1024,
+              "ring + event queue exceeds shared memory");
 
 constexpr int kMaxDevices = 64;
 
@@ -878,7 +920,7 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
   if (e != cudaSuccess) return e;
   auto set_attr = [] {
     return cudaFuncSetAttribute(k_scan_records_tma<MODE, C, STORM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)ring_smem<C>(kCtaTable<MODE, STORM>));
+                                (int)ring_smem<C>(kCtaTable<MODE, STORM>, kEq<MODE, STORM>));
   };
   if (dev < kMaxDevices) {
     std::call_once(once[dev], [&] { once_err[dev] = set_attr(); });
@@ -889,7 +931,8 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
   if (e != cudaSuccess) return e;
   // one CTA per SM; each warp a contiguous range of records (whole tiles of 32
   // where possible, so that ranges stay 512-B aligned in the header array)
-  const uint64_t warps = (uint64_t)num_sms * C::WARPS;
+  constexpr int SW = kScanWarps<MODE, C, STORM>;
+  const uint64_t warps = (uint64_t)num_sms * SW;
   Sched sch{sched_ctr, n, n, 0u, 0u, 0u, 0u, fbp.dev, fbp.host};
   uint64_t per, blocks;
   if (sched_ctr != nullptr && n >= warps * TILE * kDynMinTiles) {
@@ -909,10 +952,11 @@ cudaError_t launch_ring(const uint4* hdr, uint64_t n, const uint32_t* arena, uin
   } else {
     per = (n + warps - 1) / warps;
     per = (per + TILE - 1) / TILE * TILE;
-    blocks = ((n + per - 1) / per + C::WARPS - 1) / C::WARPS;
+    blocks = ((n + per - 1) / per + SW - 1) / SW;
   }
   if (per >= (1ull << 31)) return cudaErrorInvalidValue;  // the kernel counts a warp's records in 32 bits
-  k_scan_records_tma<MODE, C, STORM><<<(unsigned)blocks, C::WARPS * 32, ring_smem<C>(kCtaTable<MODE, STORM>), s>>>(hdr, n, arena, arena_planes,
+  k_scan_records_tma<MODE, C, STORM><<<(unsigned)blocks, C::WARPS * 32,
+                                       ring_smem<C>(kCtaTable<MODE, STORM>, kEq<MODE, STORM>), s>>>(hdr, n, arena, arena_planes,
                                                                                       base_index, per, sch, tv);
   return cudaGetLastError();
 }
@@ -1132,7 +1176,10 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   TableView tvs = tv;
   if (FPX_CAS_FIRST && !(tv.flags & FPX_OPT_NO_WARP_AGG)) tvs.flags |= TV_CAS_FIRST;
   switch (ring) {
-    case 1: return launch_ring<MODE, Ring1, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
+    case 1:
+      if constexpr (kEq<MODE, false>)
+        return launch_ring<MODE, Ring1E, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
+      return launch_ring<MODE, Ring1, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
     case 2: return launch_ring<MODE, Ring2, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
     case 3: return launch_ring<MODE, Ring3, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
     default: return launch_ring<MODE, Ring0, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
