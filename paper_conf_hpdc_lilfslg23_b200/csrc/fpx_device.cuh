@@ -201,6 +201,9 @@ static __device__ __noinline__ void table_add(const TableView tv, unsigned long 
 // one level up: per CTA instead of per warp.  A key that finds no
 // slot within CT_PROBES probes goes straight to the device table.
 constexpr uint32_t CT_SLOTS = 512, CT_PROBES = 16;
+#ifndef FPX_CT_HASH32
+#define FPX_CT_HASH32 1
+#endif
 constexpr uint32_t CT_USABLE = CT_SLOTS - 1;  // slot CT_SLOTS - 1 holds the header (see from_image)
 constexpr uint32_t CT_NONE = 0xFFFFFFFFu;
 // A tile is "dense" (its events go through the CTA table) from this many
@@ -252,7 +255,14 @@ struct CtaTable {
   }
   // one event (any lane, divergent callers welcome); c < 2^16; requires on()
   __device__ __forceinline__ void add(const TableView& tv, unsigned long long key, uint32_t c, unsigned long long f) const {
+#if FPX_CT_HASH32
+    // a 32-bit multiplicative hash mapped onto the slots with one umulhi (the
+    // 64-bit fmix + 64-bit modulo cost ~20 instructions per event in storms)
+    const uint32_t hk = ((uint32_t)(key >> 32) * 0x9E3779B1u) ^ ((uint32_t)key * 0x85EBCA77u);
+    uint32_t i = __umulhi(hk, CT_USABLE);
+#else
     uint32_t i = (uint32_t)(hash_key(key) % CT_USABLE);
+#endif
     for (uint32_t probe = 0; probe < CT_PROBES; ++probe, i = i + 1u == CT_USABLE ? 0u : i + 1u) {
       unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(keys + i);
       if (k == FPX_KEY_EMPTY) {

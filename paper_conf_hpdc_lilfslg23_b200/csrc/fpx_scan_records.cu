@@ -521,6 +521,12 @@ constexpr uint32_t kStormCap = FPX_STORM_CAP, kStormDrop = 4;
 #ifndef FPX_STORM_NO_LISTS
 #define FPX_STORM_NO_LISTS 1
 #endif
+#ifndef FPX_STORM_LEAN
+#define FPX_STORM_LEAN 1  // storm mode: one producer scan instead of two (no lists)
+#endif
+#ifndef FPX_STORM_RING
+#define FPX_STORM_RING 1
+#endif
 #ifndef FPX_STORM_START
 #define FPX_STORM_START 1
 #endif
@@ -638,13 +644,23 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     // two packed scans (full / partial active mask; byte = format).  Bytes
     // stay <= 128 over the warp, so no field overflows into the next.
     const uint32_t c8 = ni << (8 * fmt);
-    const uint32_t cf = part ? 0u : c8, cp = part ? c8 : 0u;
-    uint32_t sf = cf, sp = cp;
-    scan_step<1>(sf), scan_step<1>(sp);
-    scan_step<2>(sf), scan_step<2>(sp);
-    scan_step<4>(sf), scan_step<4>(sp);
-    scan_step<8>(sf), scan_step<8>(sp);
-    scan_step<16>(sf), scan_step<16>(sp);
+    // storm mode: the consumer skips the witnesses, so the lists are not built
+    const bool lists = !kCtaTable<MODE, STORM> || !FPX_STORM_NO_LISTS || sm.meta[0].pad[1] < kStormTiles;
+    uint32_t cf = part ? 0u : c8, cp = part ? c8 : 0u;
+    uint32_t sf, sp;
+    if (kCtaTable<MODE, STORM> && FPX_STORM_LEAN && !lists) {
+      // no lists: one scan gives the stage slots (every item counted as full)
+      cf = c8, cp = 0u;
+      sf = c8, sp = 0u;
+      scan_step<1>(sf), scan_step<2>(sf), scan_step<4>(sf), scan_step<8>(sf), scan_step<16>(sf);
+    } else {
+      sf = cf, sp = cp;
+      scan_step<1>(sf), scan_step<1>(sp);
+      scan_step<2>(sf), scan_step<2>(sp);
+      scan_step<4>(sf), scan_step<4>(sp);
+      scan_step<8>(sf), scan_step<8>(sp);
+      scan_step<16>(sf), scan_step<16>(sp);
+    }
     // a lane is in one of the two lists, so sf + sp stays <= 128 per byte
     const uint32_t incl_planes = planes_of_items(sf + sp);
     // the tile = leading records whose planes fit the stage (>= 1 record);
@@ -678,8 +694,6 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     // f's full-mask list).  Every byte stays <= 40 (items <= planes), so the
     // packed sums never carry.
     const uint32_t below = (tot_f * 0x01010101u) << 8;
-    // storm mode: the consumer skips the witnesses, so the lists are not built
-    const bool lists = !kCtaTable<MODE, STORM> || !FPX_STORM_NO_LISTS || sm.meta[0].pad[1] < kStormTiles;
     const bool writes = lists && in_tile && ni != 0u;
     uint32_t at = 0u;
     if (writes) {
@@ -1164,6 +1178,10 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   if constexpr (MODE == FPX_MODE_DEST) {
     if (storm) {  // the storm instantiation (CTA table, storm mode)
+    // storms are bound by the exact path's dependent latency (issue ~63 %):
+    // more warps per SM hide more of it, so large traces take the 24-warp
+    // ring here (FPX_STORM_RING; the sparse kernels keep Ring1)
+    if (ring == 1 && tu.ring < 0) ring = FPX_STORM_RING;
     switch (ring) {
       case 1: return launch_ring<MODE, Ring1, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
       case 2: return launch_ring<MODE, Ring2, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
