@@ -603,13 +603,16 @@ __device__ __forceinline__ bool exact_tile_transposed(const uint4 h, uint32_t ma
 // Table updates go through emit_event (the CTA pre-aggregation table, if the
 // kernel set one up, then the device table).
 // Returns whether the tile was dense (DEST transposed path, warm warp).
+// `pre`: this lane's header, already loaded by the caller (nullptr: load it).
 template <int MODE, typename Needed>
 __device__ __forceinline__ bool exact_tile_hdr(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
                                             const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
-                                            int lane, uint64_t gidx0, const TableView tv, bool warm, Needed needed) {
+                                            int lane, uint64_t gidx0, const TableView tv, bool warm, Needed needed,
+                                            const uint4* pre = nullptr) {
   if (MODE == FPX_MODE_DEST && !(tv.flags & FPX_OPT_NO_WARP_AGG)) {
     uint4 h = make_uint4(0u, 0u, 0u, 0u);
-    if ((uint32_t)lane < k) h = hdr_tile[lane];
+    if (pre != nullptr) h = *pre;
+    else if ((uint32_t)lane < k) h = hdr_tile[lane];
     const bool ok = (uint32_t)lane < k && record_valid<MODE>(h, arena_planes);
     const uint32_t mask = ok ? h.y : 0u;
     const uint32_t c = (ok && mask != 0u) ? needed(h.z) : 0u;

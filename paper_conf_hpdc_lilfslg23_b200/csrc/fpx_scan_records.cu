@@ -460,12 +460,13 @@ __device__ unsigned long long g_warp_tiles[kMaxWarpTimes], g_warp_chunks[kMaxWar
 template <int MODE>
 __device__ __forceinline__ bool exact_tile_ring(const uint4* __restrict__ hdr_tile, uint32_t k, uint64_t arena_planes,
                                                 const uint32_t* __restrict__ lane_base, const uint32_t* stage_lane,
-                                                int lane, uint64_t gidx0, const TableView tv, bool warm) {
+                                                int lane, uint64_t gidx0, const TableView tv, bool warm,
+                                                const uint4* pre = nullptr) {
   return exact_tile_hdr<MODE>(hdr_tile, k, arena_planes, lane_base, stage_lane, lane, gidx0, tv, warm, [](uint32_t meta) {
     bool f;
     const uint32_t ni = decode_items<MODE>(make_uint4(0u, FULL, meta, 0u), ~0ull, true, f, f);
     return fmt_of(meta) == FPX_FP64 ? 2u * ni : ni;
-  });
+  }, pre);
 }
 // DEST: inlined (its transposed path fits the scan loop's registers: no
 // spill).  FLOW / FLOW_DETAIL (exact_tile_flow) and the no-aggregation
@@ -523,6 +524,9 @@ constexpr uint32_t kStormCap = FPX_STORM_CAP, kStormDrop = 4;
 #endif
 #ifndef FPX_STORM_LEAN
 #define FPX_STORM_LEAN 1  // storm mode: one producer scan instead of two (no lists)
+#endif
+#ifndef FPX_STORM_HPRE
+#define FPX_STORM_HPRE 1
 #endif
 #ifndef FPX_STORM_RING
 #define FPX_STORM_RING 1
@@ -776,6 +780,14 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 #pragma unroll 1
   for (uint32_t i = 0;; ++i) {
     const int s = (int)(i % STAGES);
+    // storm kernel: the headers of the tile about to be consumed, loaded
+    // before the producer runs so that the load's latency hides behind it
+    // (every tile of a storm takes the exact path, which needs them)
+    uint4 hx = make_uint4(0u, 0u, 0u, 0u);
+    if (kCtaTable<MODE, STORM> && FPX_STORM_HPRE) {
+      const uint32_t k0 = sm.meta[s].k & ~kFlagBits;
+      hx = ld_stream4_if((uint32_t)lane < k0, hdr + (sm.meta[s].gidx0 - base_index) + lane);
+    }
     produce((int)((i + STAGES - 1) % STAGES));
     const StageMeta& m = sm.meta[s];
     const uint32_t mk = m.k;  // records in the tile | kForceBit | kNoListBit
@@ -857,7 +869,8 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
 #endif
       if (MODE == FPX_MODE_DEST && (STORM || kSparseDestCall<C> == 0)) {
         const bool dense = exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes,
-                                                 lane_base, sm.planes[s] + lane, lane, m.gidx0, tv, warm);
+                                                 lane_base, sm.planes[s] + lane, lane, m.gidx0, tv, warm,
+                                                 kCtaTable<MODE, STORM> && FPX_STORM_HPRE ? &hx : nullptr);
         if (kCtaTable<MODE, STORM> && lane == 0)
           sm.meta[0].pad[1] = dense ? min(storm_run + 1u, kStormCap) : storm_run - min(storm_run, kStormDrop);
       } else if (MODE == FPX_MODE_DEST && kSparseDestCall<C> == 1)
