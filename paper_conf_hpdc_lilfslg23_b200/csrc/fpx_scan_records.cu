@@ -420,7 +420,15 @@ constexpr uint32_t kDynChunk = 256;     // records per claimed chunk (8 tiles)
 // FLOW / FLOW_DETAIL: 128 (their tiles hold ~12 records with the sources, so
 // a 256-record chunk is ~21 tiles): C3 +0.9 % (profiles/r2/ab_flow_sched.txt)
 constexpr uint32_t kDynChunkFlow = 128;
-constexpr int kStaticPct = 75;          // share of the trace in static ranges (DEST)
+// share of the trace in static ranges (DEST).  A warp whose SM streams x
+// times slower than the average finishes its static range after the others
+// have drained the dynamic tail when x > 100 / static share: 75 % covers
+// SMs up to 1.33x slower, 60 % up to 1.67x (boxes with 1.33x SMs idle 5.5 %
+// of a C2 launch at 75 %: profiles/r2/warp_times_r2fin.txt)
+#ifndef FPX_STATIC_PCT_DEST
+#define FPX_STATIC_PCT_DEST 75
+#endif
+constexpr int kStaticPct = FPX_STATIC_PCT_DEST;
 // FLOW / FLOW_DETAIL: a smaller static share.  Some SMs stream 1.4-1.6x
 // slower than the median (tools/warp_times.py: their warps finish 255 tiles
 // of a static range while others do 313 with 15 claimed chunks), and the

@@ -9,6 +9,7 @@ import pytest
 
 import fpxgen
 import oracle
+from _mixed import sparse_flow_trace
 from _records import DEST, FP32, NAN, NONE, OP_FADD, Trace, describe_diff, entries_equal, table_dict
 
 pytestmark = pytest.mark.gpu
@@ -90,6 +91,35 @@ def test_live_option_same_table_and_every_new_key_once(fpx):
     for e in allp:  # provisional values are bounded by the final ones
         c, f = final[(int(e["site"]), int(e["fmt"]), int(e["flow"]), int(e["kind"]))]
         assert 1 <= int(e["count"]) <= c and int(e["first_index"]) >= f
+
+
+@pytest.mark.parametrize("mode", [1, 2], ids=["flow", "flow_detail"])
+def test_analyzer_live_and_fetch_new(fpx, mode):
+    """The analyzer kernels hand their table updates to the CTA's drain warp
+    (EventQueue): the table, the live ring and the FETCH_NEW windows must be
+    exactly what the scanning warps' own inserts gave -- every key once in the
+    ring and once across the FETCH_NEW windows, the table equal to the
+    oracle's."""
+    hdr, arena = sparse_flow_trace(seed=23, n=400_000)
+    d_hdr = torch.from_numpy(hdr.view(np.int32).reshape(-1, 4)).to(DEV)
+    d_arena = torch.from_numpy(arena.view(np.int32).reshape(-1)).to(DEV)
+    ref = oracle.Table()
+    ref.scan_records(hdr, arena, base_index=0, mode=mode)
+    with fpx.Handle(0, flags=fpx.OPT_LIVE_NEW) as h:
+        polled, windows = [], []
+        for a, b in ((0, 150_000), (150_000, 400_000)):
+            h.scan_records(d_hdr[a:b], d_arena, base_index=a, mode=mode, arena_planes=arena.shape[0])
+            torch.cuda.synchronize()
+            polled.append(h.poll_new(capacity=1 << 16))
+            windows.append(h.fetch_new())
+        got = h.fetch()
+    assert entries_equal(got, ref.entries()), describe_diff(got, ref.entries())
+    keys = lambda es: sorted((int(e["site"]), int(e["fmt"]), int(e["flow"]), int(e["kind"]), int(e["detail"]))
+                             for e in es)
+    allp, alln = np.concatenate(polled), np.concatenate(windows)
+    assert keys(allp) == keys(got) and len(set(keys(allp))) == len(allp)
+    assert keys(alln) == keys(got) and len(set(keys(alln))) == len(alln)
+    assert {int(e["flow"]) for e in got} == {1, 2, 3}
 
 
 def test_poll_without_option_is_invalid(fpx):

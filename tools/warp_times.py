@@ -12,6 +12,16 @@ import os
 import subprocess
 import sys
 
+# One config per process: the per-warp arrays are device globals indexed by
+# scan warp, and kernels with different scan-warp counts (the analyzer's drain
+# warp) would otherwise read another config's stale entries.
+_CFGS = sys.argv[1:] or ["c2", "c3", "c4a", "c5"]
+if len(_CFGS) > 1:
+    for _c in _CFGS:
+        sys.stdout.flush()
+        subprocess.run([sys.executable, os.path.abspath(__file__), _c], check=False)
+    sys.exit(0)
+
 import numpy as np
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -38,7 +48,7 @@ wt = ctypes.CDLL(LIB)
 wt.fpx_debug_warp_times.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int]
 NW = 148 * 32
 
-for name in sys.argv[1:] or ["c2", "c3", "c4a", "c5"]:
+for name in _CFGS:
     cfg = dict(bench.CONFIGS[name])
     wl = bench.RecordsWorkload(cfg, 0, bench.config_seed(name), "tma")
     stream = torch.cuda.current_stream()
