@@ -533,6 +533,9 @@ constexpr uint32_t kStormCap = FPX_STORM_CAP, kStormDrop = 4;
 #ifndef FPX_STORM_LEAN
 #define FPX_STORM_LEAN 1  // storm mode: one producer scan instead of two (no lists)
 #endif
+#ifndef FPX_DEST_RING
+#define FPX_DEST_RING 1  // the sparse DEST kernels' ring for large traces (1: Ring1, 4: Ring4)
+#endif
 #ifndef FPX_STORM_HPRE
 #define FPX_STORM_HPRE 1
 #endif
@@ -933,9 +936,13 @@ using Ring3 = RingCfg<24, 2, 32>;
 // the analyzer kernels with the drain warp (kEq): 19 scan warps x 42 planes
 // keep Ring1's bytes in flight
 using Ring1E = RingCfg<20, 2, 42>;
+// 18 warps x 46 planes (A/B: FPX_DEST_RING=4): tiles of mixed FP32 / FP64
+// records reach 32 records (C2 averages ~26 per 40-plane tile)
+using Ring4 = RingCfg<18, 2, 46>;
 static_assert(sizeof(WarpSmem<Ring2>) % 128 == 0 && ring_smem<Ring0>() <= 227 * 1024 && ring_smem<Ring1>() <= 227 * 1024 &&
                   ring_smem<Ring2>() <= 227 * 1024 && ring_smem<Ring3>() <= 227 * 1024,
               "ring exceeds shared memory");
+static_assert(ring_smem<Ring4>(false) <= 227 * 1024, "ring 4 exceeds shared memory");
 static_assert(ring_smem<Ring0>(false, true) <= 227 * 1024 && ring_smem<Ring1E>(false, true) <= 227 * 1024 &&
                   ring_smem<Ring2>(false, true) <= 227 * 1024 && ring_smem<Ring3>(false, true) <= 227 * 1024,
               "ring + event queue exceeds shared memory");
@@ -1191,7 +1198,7 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   // decides.
   const Tuning& tu = tuning();
   int ring = tu.ring;
-  if (ring < 0) ring = n <= (uint64_t)num_sms * 24 * TILE ? 3 : 1;
+  if (ring < 0) ring = n <= (uint64_t)num_sms * 24 * TILE ? 3 : MODE == FPX_MODE_DEST ? FPX_DEST_RING : 1;
   if (tu.sched == 0) sched_ctr = nullptr;
   const int static_pct = tu.static_pct >= 0 ? tu.static_pct : MODE == FPX_MODE_DEST ? kStaticPct : kStaticPctFlow;
   const uint32_t chunk = tu.dyn_chunk ? tu.dyn_chunk : MODE == FPX_MODE_DEST ? kDynChunk : kDynChunkFlow;
@@ -1199,9 +1206,9 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   if constexpr (MODE == FPX_MODE_DEST) {
     if (storm) {  // the storm instantiation (CTA table, storm mode)
-    // storms are bound by the exact path's dependent latency (issue ~63 %):
-    // more warps per SM hide more of it, so large traces take the 24-warp
-    // ring here (FPX_STORM_RING; the sparse kernels keep Ring1)
+    // large traces: Ring1 (FPX_STORM_RING; the 24-warp Ring3 lost 6 % on
+    // both storms: profiles/r2/ab_storm_ring.txt)
+    if (ring == 4) ring = 1;
     if (ring == 1 && tu.ring < 0) ring = FPX_STORM_RING;
     switch (ring) {
       case 1: return launch_ring<MODE, Ring1, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
@@ -1221,6 +1228,10 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
       return launch_ring<MODE, Ring1, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
     case 2: return launch_ring<MODE, Ring2, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
     case 3: return launch_ring<MODE, Ring3, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
+    case 4:
+      if constexpr (MODE == FPX_MODE_DEST && FPX_DEST_RING == 4)
+        return launch_ring<MODE, Ring4, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
+      [[fallthrough]];
     default: return launch_ring<MODE, Ring0, false>(h4, n, d_arena, arena_planes, base_index, tvs, num_sms, sched_ctr, scfg, fbp, s);
   }
 }
