@@ -206,6 +206,10 @@ constexpr uint32_t CT_SLOTS = 512, CT_PROBES = 16;
 #endif
 constexpr uint32_t CT_USABLE = CT_SLOTS - 1;  // slot CT_SLOTS - 1 holds the header (see from_image)
 constexpr uint32_t CT_NONE = 0xFFFFFFFFu;
+constexpr uint32_t CT_ON = 1u, CT_ON_RED = 2u;  // the header's "on" word
+#ifndef FPX_CT_RED
+#define FPX_CT_RED 1
+#endif
 // A tile is "dense" (its events go through the CTA table) from this many
 // warp-reduced events (FLOW / pending batches) or records with an event
 // (DEST transposed path) on.
@@ -219,6 +223,7 @@ struct CtaTable {
                              // and the first offsets [CT_SLOTS] (u32, min first index - base);
                              // nullptr: no CTA table (events go to the device table)
   unsigned long long base;   // the launch's base index
+  bool red = false;          // counts by RED (no returned value, no drain): see init
   __host__ __device__ static constexpr size_t bytes() { return CT_SLOTS * 16; }
   __device__ __forceinline__ unsigned int* cnt() const { return reinterpret_cast<unsigned int*>(keys + CT_SLOTS); }
   __device__ __forceinline__ unsigned int* first() const { return cnt() + CT_SLOTS; }
@@ -238,10 +243,13 @@ struct CtaTable {
     uint8_t* smem = image_at();
     const unsigned long long* k = reinterpret_cast<const unsigned long long*>(smem);
     const unsigned int* c = reinterpret_cast<const unsigned int*>(k + CT_SLOTS);
-    return CtaTable{c[CT_USABLE] ? reinterpret_cast<unsigned long long*>(smem) : nullptr, k[CT_USABLE]};
+    return CtaTable{c[CT_USABLE] ? reinterpret_cast<unsigned long long*>(smem) : nullptr, k[CT_USABLE],
+                    c[CT_USABLE] == CT_ON_RED};
   }
-  // by the whole CTA, before a __syncthreads
-  __device__ void init(bool on_) const {
+  // by the whole CTA, before a __syncthreads.  red_ok: the launch has fewer
+  // than 2^24 records, so no slot's count (<= 256 lane-values per record)
+  // can reach 2^32: counts are added with a fire-and-forget shared reduction
+  __device__ void init(bool on_, bool red_ok = false) const {
     for (uint32_t i = threadIdx.x; i < CT_USABLE; i += blockDim.x) {
       keys[i] = FPX_KEY_EMPTY;
       cnt()[i] = 0u;
@@ -249,7 +257,7 @@ struct CtaTable {
     }
     if (threadIdx.x == 0) {
       keys[CT_USABLE] = base;
-      cnt()[CT_USABLE] = on_ ? 1u : 0u;
+      cnt()[CT_USABLE] = !on_ ? 0u : red_ok ? CT_ON_RED : CT_ON;
       first()[CT_USABLE] = 0u;  // warps done (cta_warp_done)
     }
   }
@@ -277,6 +285,10 @@ struct CtaTable {
         unsigned int* ci = cnt() + i;
         const uint32_t off = (uint32_t)(f - base);
         if (off < *reinterpret_cast<volatile unsigned int*>(fi)) atomicMin(fi, off);
+        if (red) {  // nothing to wait for (S1 / S2: ab_ct_red.txt)
+          asm volatile("red.shared.add.u32 [%0], %1;" ::"r"((uint32_t)__cvta_generic_to_shared(ci)), "r"(c) : "memory");
+          return;
+        }
         const uint32_t old = atomicAdd(ci, c);
         if (old + c >= 0x80000000u) {  // keep the 32-bit count far from overflow: drain it
           const uint32_t v = atomicExch(ci, 0u);

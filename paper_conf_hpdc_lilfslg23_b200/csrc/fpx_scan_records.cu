@@ -570,7 +570,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   // than 32 bits
   if (kCtaTable<MODE, STORM>)
     CtaTable{reinterpret_cast<unsigned long long*>(CtaTable::image_at()), base_index}
-        .init((tv.flags & FPX_OPT_NO_WARP_AGG) == 0u && n < (uint64_t)CT_NONE);
+        .init((tv.flags & FPX_OPT_NO_WARP_AGG) == 0u && n < (uint64_t)CT_NONE, FPX_CT_RED && n < (1ull << 24));
   if (kEq<MODE, STORM>) EventQueue::from_image().init();
   __syncthreads();
   constexpr int SW = kScanWarps<MODE, C, STORM>;
