@@ -536,8 +536,18 @@ constexpr uint32_t kStormCap = FPX_STORM_CAP, kStormDrop = 4;
 #ifndef FPX_DEST_RING
 #define FPX_DEST_RING 1  // the sparse DEST kernels' ring for large traces (1: Ring1, 4: Ring4)
 #endif
+// BF16 items go into the FP16 lists and take the FP16 witness, which never
+// misses a BF16 exception: a doubled BF16 half is subnormal iff it lies in
+// [2, 0xFF] (inside FP16's [2, 0x7FF]) and INF / NaN iff >= 0xFF00 (inside
+// FP16's >= 0xF800).  Its false positives are BF16 values below 2^-119 or
+// above 2^120 in magnitude, which a hit tile's exact path then finds clean.
+// Two list loops fewer per tile of packed records (C4a: ab_merge_halves.txt).
+#ifndef FPX_MERGE_HALVES
+#define FPX_MERGE_HALVES 1
+#endif
+constexpr bool kMergeHalves = FPX_MERGE_HALVES != 0;
 #ifndef FPX_STORM_HPRE
-#define FPX_STORM_HPRE 1
+#define FPX_STORM_HPRE 1  // 1: loaded before the producer of the same iteration, 2: one iteration ahead (S1 / S2 -3.5 %: ab_storm_hpre.txt)
 #endif
 #ifndef FPX_STORM_RING
 #define FPX_STORM_RING 1
@@ -658,7 +668,9 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     const bool part = mask != FULL;
     // two packed scans (full / partial active mask; byte = format).  Bytes
     // stay <= 128 over the warp, so no field overflows into the next.
-    const uint32_t c8 = ni << (8 * fmt);
+    // list format: BF16 items share the FP16 lists (kMergeHalves)
+    const uint32_t lfmt = kMergeHalves ? min(fmt, (uint32_t)FPX_FP16) : fmt;
+    const uint32_t c8 = ni << (8 * lfmt);
     // storm mode: the consumer skips the witnesses, so the lists are not built
     const bool lists = !kCtaTable<MODE, STORM> || !FPX_STORM_NO_LISTS || sm.meta[0].pad[1] < kStormTiles;
     uint32_t cf = part ? 0u : c8, cp = part ? c8 : 0u;
@@ -714,7 +726,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     if (writes) {
       // byte f of `own`: this record's place among format f's items (full list first)
       const uint32_t own = part ? tf + (sp - cp) : sf - cf;
-      at = ((below + own) >> (8 * fmt)) & 0xFFu;
+      at = ((below + own) >> (8 * lfmt)) & 0xFFu;
       sm.items[s][at] = make_uint2(slot, mask);
     }
 #ifndef FPX_ITEMS_PREDICATED
@@ -788,6 +800,17 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
   uint32_t phase = 0;  // bit s = parity to wait for on stage s
 #pragma unroll 1
   for (int s = 0; s < STAGES - 1; ++s) produce(s);
+  // storm kernel, FPX_STORM_HPRE 2: the exact path's headers of the tile
+  // consumed next, loaded one loop iteration ahead (the first use of the
+  // headers loaded before the producer was still 7.7 % of S2's stall samples,
+  // r2v15) -- but holding them across the loop spills: S1 / S2 -3.5 %, so the
+  // default stays 1 (ab_storm_hpre.txt)
+  auto load_hx = [&](int st) {
+    const uint32_t k0 = sm.meta[st].k & ~kFlagBits;
+    return ld_stream4_if((uint32_t)lane < k0, hdr + (sm.meta[st].gidx0 - base_index) + lane);
+  };
+  uint4 hx_next = make_uint4(0u, 0u, 0u, 0u);
+  if (kCtaTable<MODE, STORM> && FPX_STORM_HPRE == 2) hx_next = load_hx(0);
 #pragma unroll 1
   for (uint32_t i = 0;; ++i) {
     const int s = (int)(i % STAGES);
@@ -795,11 +818,12 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     // before the producer runs so that the load's latency hides behind it
     // (every tile of a storm takes the exact path, which needs them)
     uint4 hx = make_uint4(0u, 0u, 0u, 0u);
-    if (kCtaTable<MODE, STORM> && FPX_STORM_HPRE) {
-      const uint32_t k0 = sm.meta[s].k & ~kFlagBits;
-      hx = ld_stream4_if((uint32_t)lane < k0, hdr + (sm.meta[s].gidx0 - base_index) + lane);
-    }
+    if (kCtaTable<MODE, STORM> && FPX_STORM_HPRE == 1) hx = load_hx(s);
     produce((int)((i + STAGES - 1) % STAGES));
+    if (kCtaTable<MODE, STORM> && FPX_STORM_HPRE == 2) {
+      hx = hx_next;
+      hx_next = load_hx((int)((i + 1) % STAGES));
+    }
     const StageMeta& m = sm.meta[s];
     const uint32_t mk = m.k;  // records in the tile | kForceBit | kNoListBit
     if (mk == 0u) {
@@ -860,11 +884,16 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       consume_list<FPX_FP64, true>(w, byte_of(sp, 1), s2, ia, pa, g, q);
       const bool halves = s2 != tot;
       if (halves) {
-        const uint32_t s3 = byte_of(sb, 3);
-        consume_list<FPX_FP16, false>(w, s2, byte_of(sp, 2), ia, pa, g, q);
-        consume_list<FPX_FP16, true>(w, byte_of(sp, 2), s3, ia, pa, g, q);
-        consume_list<FPX_BF16, false>(w, s3, byte_of(sp, 3), ia, pa, g, q);
-        consume_list<FPX_BF16, true>(w, byte_of(sp, 3), tot, ia, pa, g, q);
+        if (kMergeHalves) {
+          consume_list<FPX_FP16, false>(w, s2, byte_of(sp, 2), ia, pa, g, q);
+          consume_list<FPX_FP16, true>(w, byte_of(sp, 2), tot, ia, pa, g, q);
+        } else {
+          const uint32_t s3 = byte_of(sb, 3);
+          consume_list<FPX_FP16, false>(w, s2, byte_of(sp, 2), ia, pa, g, q);
+          consume_list<FPX_FP16, true>(w, byte_of(sp, 2), s3, ia, pa, g, q);
+          consume_list<FPX_BF16, false>(w, s3, byte_of(sp, 3), ia, pa, g, q);
+          consume_list<FPX_BF16, true>(w, byte_of(sp, 3), tot, ia, pa, g, q);
+        }
       }
       hit = __any_sync(FULL, w.hit_wide() || (halves && w.hit_half())) || (mk & kForceBit) != 0u;
     }
