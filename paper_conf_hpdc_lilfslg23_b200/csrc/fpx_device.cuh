@@ -323,7 +323,15 @@ static __device__ __noinline__ void emit_event(const TableView tv, unsigned long
 // A record's per-kind counts (16 bits per kind in cnt, kinds in `present`)
 // straight into the CTA table (warm warps, dense tiles of the transposed
 // DEST path); out of line like emit_event.
-static __device__ __noinline__ void emit_kinds_cta(const TableView tv, uint32_t site, uint32_t fmt, uint32_t present,
+#ifndef FPX_EMIT_INLINE
+#define FPX_EMIT_INLINE 0
+#endif
+#if FPX_EMIT_INLINE
+static __device__ __forceinline__
+#else
+static __device__ __noinline__
+#endif
+void emit_kinds_cta(const TableView tv, uint32_t site, uint32_t fmt, uint32_t present,
                                                   unsigned long long cnt, unsigned long long f) {
   const CtaTable ct = CtaTable::from_image();
   while (present) {
