@@ -579,6 +579,22 @@ def test_fetch_new_truncated_windows_lose_nothing(fpx):
         assert [int(e["site"]) for e in h.fetch_new(capacity=30)] == [500]
 
 
+@pytest.mark.parametrize("dense", [1.0, 0.01])
+def test_storm_cta_large_launch(fpx, dense):
+    """A storm launch of more than 2^24 records: the CTA table then adds its
+    counts with the returning atomic and drains a slot before 2^31 (below
+    2^24 records it uses a shared reduction, which cannot overflow there);
+    the table must still equal the oracle's."""
+    n = (1 << 24) + 4099
+    p = fpxgen.Params(seed=90, n_records=n, n_sites=200, recipe=fpxgen.RECIPE_STRESS, dense_nan=dense)
+    hdr, arena = fpxgen.generate_host(p)
+    base = 11
+    exp = oracle_scan(hdr, arena, base, DEST).entries()
+    got, st, _ = gpu_scan(fpx, hdr, arena, base=base, mode=DEST, flags=fpx.OPT_STORM)
+    assert st == fpx.OK
+    assert_same(got, exp)
+
+
 @pytest.mark.parametrize("mode", [DEST, FLOW, FLOW_DETAIL])
 @pytest.mark.parametrize("dense", [1.0, 0.01])
 def test_storm_cta_preaggregation(fpx, mode, dense):
