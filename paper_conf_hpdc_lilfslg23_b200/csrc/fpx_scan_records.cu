@@ -98,9 +98,10 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 // ---- TMA-ring kernel ------------------------------------------------------------
 // Ring geometry: WARPS warps per CTA (one CTA per SM), STAGES stages per warp
 // (STAGES-1 tiles in flight while one is consumed), PLANES planes per stage.
-template <int WARPS_, int STAGES_, int PLANES_>
+template <int WARPS_, int STAGES_, int PLANES_, bool STASH_ = false>
 struct RingCfg {
   static constexpr int WARPS = WARPS_, STAGES = STAGES_, PLANES = PLANES_;
+  static constexpr bool STASH = STASH_;  // the producer keeps each tile's headers in shared memory
 };
 
 // Fast-path item lists of a stage: 4 formats x {full, partial active mask}.
@@ -128,6 +129,7 @@ struct alignas(128) WarpSmem {  // 128-B multiple: every warp's planes stay 16-B
   uint2 items[C::STAGES][C::PLANES];           // {plane slot, active mask}
   StageMeta meta[C::STAGES];
   uint64_t bar[C::STAGES];
+  uint4 hdrs[C::STASH ? C::STAGES : 1][C::STASH ? 32 : 1];  // STASH: the tile's headers (lane = record)
 };
 // Header-decode table, one byte per (opclass < 32, fmt, nsrc, dwords):
 // low nibble = fast-path items (0..4), DECODE_FORCE (DIV: exact path) or
@@ -550,7 +552,7 @@ constexpr bool kMergeHalves = FPX_MERGE_HALVES != 0;
 #define FPX_STORM_HPRE 1  // 1: loaded before the producer of the same iteration, 2: one iteration ahead (S1 / S2 -3.5 %: ab_storm_hpre.txt)
 #endif
 #ifndef FPX_STORM_RING
-#define FPX_STORM_RING 1
+#define FPX_STORM_RING 5  // Ring5: 36-plane stages + header stash (S1 +3.0 %, S2 +3.4 %: ab_storm_stash.txt)
 #endif
 #ifndef FPX_STORM_START
 #define FPX_STORM_START 1
@@ -660,6 +662,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       return;
     }
     const bool inrange = (uint32_t)lane < rem;
+    if (C::STASH) sm.hdrs[s][lane] = h;  // the exact path reads them from here (no L2 reload)
     bool ok, force;
     uint32_t foot_all;
     const uint32_t ni = decode_fast(lut, h, arena_planes, inrange, ok, force, foot_all);
@@ -818,7 +821,7 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
     // before the producer runs so that the load's latency hides behind it
     // (every tile of a storm takes the exact path, which needs them)
     uint4 hx = make_uint4(0u, 0u, 0u, 0u);
-    if (kCtaTable<MODE, STORM> && FPX_STORM_HPRE == 1) hx = load_hx(s);
+    if (kCtaTable<MODE, STORM> && FPX_STORM_HPRE == 1 && !C::STASH) hx = load_hx(s);
     produce((int)((i + STAGES - 1) % STAGES));
     if (kCtaTable<MODE, STORM> && FPX_STORM_HPRE == 2) {
       hx = hx_next;
@@ -908,9 +911,10 @@ k_scan_records_tma(const uint4* __restrict__ hdr, uint64_t n, const uint32_t* __
       const uint64_t te0 = globaltimer_ns();
 #endif
       if (MODE == FPX_MODE_DEST && (STORM || kSparseDestCall<C> == 0)) {
+        if (C::STASH) hx = sm.hdrs[s][lane];
         const bool dense = exact_tile_ring<MODE>(hdr + (m.gidx0 - base_index), mk & ~kFlagBits, arena_planes,
                                                  lane_base, sm.planes[s] + lane, lane, m.gidx0, tv, warm,
-                                                 kCtaTable<MODE, STORM> && FPX_STORM_HPRE ? &hx : nullptr);
+                                                 kCtaTable<MODE, STORM> && (FPX_STORM_HPRE || C::STASH) ? &hx : nullptr);
         if (kCtaTable<MODE, STORM> && lane == 0)
           sm.meta[0].pad[1] = dense ? min(storm_run + 1u, kStormCap) : storm_run - min(storm_run, kStormDrop);
       } else if (MODE == FPX_MODE_DEST && kSparseDestCall<C> == 1)
@@ -965,6 +969,12 @@ using Ring3 = RingCfg<24, 2, 32>;
 // the analyzer kernels with the drain warp (kEq): 19 scan warps x 42 planes
 // keep Ring1's bytes in flight
 using Ring1E = RingCfg<20, 2, 42>;
+// the storm kernel (FPX_STORM_RING 5): Ring1's warps with 36-plane stages and
+// the tiles' headers kept in the freed shared memory, so the exact path,
+// which every storm tile takes, reads them with LDS instead of reloading
+// them from L2 (the first use of the reloaded headers was 7.7 % of S2's stall
+// samples, r2v15); one-plane storm tiles use 32 planes anyway
+using Ring5 = RingCfg<20, 2, 36, true>;
 // 18 warps x 46 planes (A/B: FPX_DEST_RING=4): tiles of mixed FP32 / FP64
 // records reach 32 records (C2 averages ~26 per 40-plane tile)
 using Ring4 = RingCfg<18, 2, 46>;
@@ -972,6 +982,7 @@ static_assert(sizeof(WarpSmem<Ring2>) % 128 == 0 && ring_smem<Ring0>() <= 227 * 
                   ring_smem<Ring2>() <= 227 * 1024 && ring_smem<Ring3>() <= 227 * 1024,
               "ring exceeds shared memory");
 static_assert(ring_smem<Ring4>(false) <= 227 * 1024, "ring 4 exceeds shared memory");
+static_assert(ring_smem<Ring5>(true) <= 227 * 1024, "ring 5 exceeds shared memory");
 static_assert(ring_smem<Ring0>(false, true) <= 227 * 1024 && ring_smem<Ring1E>(false, true) <= 227 * 1024 &&
                   ring_smem<Ring2>(false, true) <= 227 * 1024 && ring_smem<Ring3>(false, true) <= 227 * 1024,
               "ring + event queue exceeds shared memory");
@@ -1235,12 +1246,14 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   const uint4* h4 = reinterpret_cast<const uint4*>(d_hdr);
   if constexpr (MODE == FPX_MODE_DEST) {
     if (storm) {  // the storm instantiation (CTA table, storm mode)
-    // large traces: Ring1 (FPX_STORM_RING; the 24-warp Ring3 lost 6 % on
-    // both storms: profiles/r2/ab_storm_ring.txt)
+    // large traces: Ring5, 36-plane stages with the headers stashed in shared
+    // memory (FPX_STORM_RING; the 24-warp Ring3 lost 6 % on both storms:
+    // profiles/r2/ab_storm_ring.txt)
     if (ring == 4) ring = 1;
     if (ring == 1 && tu.ring < 0) ring = FPX_STORM_RING;
     switch (ring) {
       case 1: return launch_ring<MODE, Ring1, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
+      case 5: return launch_ring<MODE, Ring5, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
       case 2: return launch_ring<MODE, Ring2, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
       case 3: return launch_ring<MODE, Ring3, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
       default: return launch_ring<MODE, Ring0, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
