@@ -307,13 +307,17 @@ __device__ __forceinline__ void count4_fp32(const uint4 x, uint32_t m4, uint32_t
 #ifndef FPX_COUNT_FP
 #define FPX_COUNT_FP 1
 #endif
+#ifndef FPX_COUNT_UNROLL
+#define FPX_COUNT_UNROLL 4  // quads per unrolled step of the transposed class count
+#endif
+constexpr int kCountUnroll = FPX_COUNT_UNROLL;
 
 template <uint32_t FMT>
 __device__ __forceinline__ void count_staged(uint32_t sp, uint32_t dw, uint32_t mask, uint32_t lane, uint32_t& n_nan,
                                              uint32_t& n_inf, uint32_t& n_sub) {
   constexpr uint32_t STEP = FMT == FPX_FP64 ? 2u : 1u;
   for (uint32_t w = 0; w < dw; w += STEP) {
-#pragma unroll 4
+#pragma unroll kCountUnroll
     for (uint32_t u = 0; u < 8; ++u) {
       const uint32_t v = (u + lane) & 7u;
       const uint32_t m4 = mask >> (4u * v);
