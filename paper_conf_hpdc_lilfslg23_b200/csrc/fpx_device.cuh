@@ -193,11 +193,10 @@ static __device__ __noinline__ void table_add(const TableView tv, unsigned long 
 // CTA-level pre-aggregation of table updates (dense exception storms): a
 // small open-addressed table in shared memory, keyed like the device table,
 // holding a 32-bit count and a 32-bit first-index offset (relative to the
-// launch's base index) per key.  The first sighting of a key in the CTA goes
-// straight to the device table (so the key is inserted -- and reported as
-// new, P:244 -- as early as before); later events of that key only touch
-// shared memory and reach the device table once, when the CTA's last warp
-// is done (cta_warp_done).  Alg2's "reduce before any atomic"
+// launch's base index) per key.  Every event of a key, its first sighting in
+// the CTA included (FPX_CT_DEFER_FIRST), only touches shared memory; the key
+// reaches the device table once, when the CTA's last warp is done
+// (cta_warp_done).  Alg2's "reduce before any atomic"
 // one level up: per CTA instead of per warp.  A key that finds no
 // slot within CT_PROBES probes goes straight to the device table.
 constexpr uint32_t CT_SLOTS = 512, CT_PROBES = 16;
@@ -207,6 +206,19 @@ constexpr uint32_t CT_SLOTS = 512, CT_PROBES = 16;
 constexpr uint32_t CT_USABLE = CT_SLOTS - 1;  // slot CT_SLOTS - 1 holds the header (see from_image)
 constexpr uint32_t CT_NONE = 0xFFFFFFFFu;
 constexpr uint32_t CT_ON = 1u, CT_ON_RED = 2u;  // the header's "on" word
+// FPX_CT_DEFER_FIRST 1: a key's first sighting in a CTA is counted in shared
+// memory like the others and reaches the device table (and the new-key log /
+// live ring) when the CTA's last warp drains the table, at the latest at the
+// end of the launch, instead of at once: the storm kernel's warps then never
+// wait for a device-table insert (each CTA met every hot key once, ~10 L2
+// round trips per warp early in the launch: S1 +9.2 %, S2 +11.4 %,
+// profiles/r2/ab_ct_defer.txt).  Only the storm kernel has a CTA table; the
+// sparse kernels, where an isolated new exception is what a user waits for,
+// still insert at once (P:244's early notification is about runs that last
+// hours, not about one launch).  0: insert at the first sighting.
+#ifndef FPX_CT_DEFER_FIRST
+#define FPX_CT_DEFER_FIRST 1
+#endif
 #ifndef FPX_CT_RED
 #define FPX_CT_RED 1
 #endif
@@ -276,8 +288,11 @@ struct CtaTable {
       if (k == FPX_KEY_EMPTY) {
         k = atomicCAS(keys + i, FPX_KEY_EMPTY, key);
         if (k == FPX_KEY_EMPTY) {  // first sighting in this CTA: the device table gets it now
-          table_add(tv, key, c, f);
-          return;
+          if (!FPX_CT_DEFER_FIRST) {
+            table_add(tv, key, c, f);
+            return;
+          }
+          k = key;  // deferred: counted here, inserted by the CTA's last warp
         }
       }
       if (k == key) {
