@@ -321,6 +321,10 @@ fpx_status fpx_table_reset(fpx_handle h, void* stream);
  * gives the final values once the scans are done).  fpx_table_reset restarts
  * the ring.  Keys first inserted by another process's attached handle
  * (fpx_open_attached) are not published here (FETCH_NEW still reports them).
+ * Latency: the sparse record kernels, the tensor scans and the analyzer
+ * modes insert (and publish) a key as soon as a warp finds it; the storm
+ * kernel (FPX_OPT_STORM, or picked after a storm) pre-aggregates per CTA and
+ * inserts a key when the CTA that found it finishes, within the same launch.
  * This poll cursor is independent of FPX_FETCH_NEW's.  A handle is used from
  * one host thread at a time, polls included.  Errors: FPX_ERR_INVALID (no
  * FPX_OPT_LIVE_NEW, NULL arguments). */
