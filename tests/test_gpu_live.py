@@ -65,9 +65,12 @@ def test_poll_sees_planted_key_before_the_scans_finish(fpx):
         assert len(again) == 1 and int(again[0]["first_index"]) == 10 + r
 
 
-def test_live_option_same_table_and_every_new_key_once(fpx):
+@pytest.mark.parametrize("storm", [False, True], ids=["sparse", "storm"])
+def test_live_option_same_table_and_every_new_key_once(fpx, storm):
     """With FPX_OPT_LIVE_NEW the fetched table equals the oracle's and every
-    key is polled exactly once across batches (poll keys == FETCH_ALL keys)."""
+    key is polled exactly once across batches (poll keys == FETCH_ALL keys);
+    also through the storm kernel, which inserts a CTA's new keys when the
+    CTA finishes."""
     p = fpxgen.Params(seed=9, n_records=300_000, n_sites=5000, recipe=fpxgen.RECIPE_MIX)
     hdr, arena = fpxgen.generate_host(p)
     _, w = fpxgen.plan_injections(p, 3000)
@@ -76,7 +79,7 @@ def test_live_option_same_table_and_every_new_key_once(fpx):
     d_arena = torch.from_numpy(arena.view(np.int32).reshape(-1)).to(DEV)
     ref = oracle.Table()
     ref.scan_records(hdr, arena, base_index=0)
-    with fpx.Handle(0, flags=fpx.OPT_LIVE_NEW) as h:
+    with fpx.Handle(0, flags=fpx.OPT_LIVE_NEW | (fpx.OPT_STORM if storm else 0)) as h:
         polled = []
         for a, b in ((0, 100_000), (100_000, 300_000)):
             h.scan_records(d_hdr[a:b], d_arena, base_index=a, arena_planes=arena.shape[0])
