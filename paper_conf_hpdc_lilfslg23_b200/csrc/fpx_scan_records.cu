@@ -548,6 +548,9 @@ constexpr uint32_t kStormCap = FPX_STORM_CAP, kStormDrop = 4;
 #define FPX_MERGE_HALVES 1
 #endif
 constexpr bool kMergeHalves = FPX_MERGE_HALVES != 0;
+#ifndef FPX_ONE_PLANE_RING
+#define FPX_ONE_PLANE_RING 1
+#endif
 #ifndef FPX_STORM_HPRE
 #define FPX_STORM_HPRE 1  // 1: loaded before the producer of the same iteration, 2: one iteration ahead (S1 / S2 -3.5 %: ab_storm_hpre.txt)
 #endif
@@ -1238,7 +1241,15 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
   // decides.
   const Tuning& tu = tuning();
   int ring = tu.ring;
-  if (ring < 0) ring = n <= (uint64_t)num_sms * 24 * TILE ? 3 : MODE == FPX_MODE_DEST ? FPX_DEST_RING : 1;
+  const bool small = n <= (uint64_t)num_sms * 24 * TILE;
+  // one-plane DEST traces (an arena of at most 1.1 planes per record: FP32 /
+  // packed scalar ops) fill only 32 of a 40-plane stage -- a tile holds at
+  // most 32 records -- so they take the 24-warp x 32-plane ring: 20 % more
+  // bytes in flight (C5 +2.1 %; multi-plane traces lose 3-6 % on it, C2 /
+  // C4a: profiles/r2/ab_dest_ring3.txt).  Host-side, from the call's own
+  // arguments; an arena with other data in it only keeps the default ring.
+  const bool one_plane = MODE == FPX_MODE_DEST && FPX_ONE_PLANE_RING && arena_planes * 10 <= n * 11;
+  if (ring < 0) ring = small || one_plane ? 3 : MODE == FPX_MODE_DEST ? FPX_DEST_RING : 1;
   if (tu.sched == 0) sched_ctr = nullptr;
   const int static_pct = tu.static_pct >= 0 ? tu.static_pct : MODE == FPX_MODE_DEST ? kStaticPct : kStaticPctFlow;
   const uint32_t chunk = tu.dyn_chunk ? tu.dyn_chunk : MODE == FPX_MODE_DEST ? kDynChunk : kDynChunkFlow;
@@ -1249,8 +1260,7 @@ cudaError_t launch_records_t(const fpx_rec_hdr* d_hdr, uint64_t n, const uint32_
     // large traces: Ring5, 36-plane stages with the headers stashed in shared
     // memory (FPX_STORM_RING; the 24-warp Ring3 lost 6 % on both storms:
     // profiles/r2/ab_storm_ring.txt)
-    if (ring == 4) ring = 1;
-    if (ring == 1 && tu.ring < 0) ring = FPX_STORM_RING;
+    if (tu.ring < 0) ring = small ? 3 : FPX_STORM_RING;
     switch (ring) {
       case 1: return launch_ring<MODE, Ring1, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
       case 5: return launch_ring<MODE, Ring5, true>(h4, n, d_arena, arena_planes, base_index, tv, num_sms, sched_ctr, scfg, fbp, s);
